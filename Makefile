@@ -1,0 +1,33 @@
+# Native build: every .so is built in-tree (they travel to the GPU box with gpurun).
+#   graphgen/libgraphgen.so                 seeded input generators (CPU + CUDA)
+#   oracle/liboracle.so                     plain-C CPU oracle (test infrastructure only)
+#   paper_conf_sigmod_hu0l21_b200/libtc_b200.so   the product: C-ABI + sm_100a kernels
+NVCC    ?= /usr/local/cuda/bin/nvcc
+CC      ?= gcc
+ARCH    := -gencode arch=compute_100a,code=sm_100a
+NVFLAGS := $(ARCH) -O3 -lineinfo -std=c++17 -Xcompiler -fPIC -Xcompiler -Wall \
+           -Xptxas -v --expt-relaxed-constexpr
+CFLAGS  := -O2 -std=c11 -fPIC -Wall -Wextra -ffp-contract=off
+
+PKG := paper_conf_sigmod_hu0l21_b200
+TC_SRCS := $(wildcard $(PKG)/csrc/*.cu)
+TC_HDRS := $(wildcard $(PKG)/csrc/*.cuh) include/tc.h
+TC_CPP  := $(wildcard $(PKG)/csrc/*.cpp)
+
+all: graphgen/libgraphgen.so oracle/liboracle.so $(PKG)/libtc_b200.so
+
+graphgen/libgraphgen.so: graphgen/graphgen_cpu.c graphgen/graphgen_cuda.cu graphgen/philox.h
+	$(CC) $(CFLAGS) -c graphgen/graphgen_cpu.c -o graphgen/graphgen_cpu.o
+	$(NVCC) $(ARCH) -O3 -Xcompiler -fPIC -c graphgen/graphgen_cuda.cu -o graphgen/graphgen_cuda.o
+	$(NVCC) $(ARCH) -shared graphgen/graphgen_cpu.o graphgen/graphgen_cuda.o -o $@ -lpthread
+
+oracle/liboracle.so: oracle/tc_oracle.c
+	$(CC) $(CFLAGS) -shared oracle/tc_oracle.c -o $@ -lm
+
+$(PKG)/libtc_b200.so: $(TC_SRCS) $(TC_HDRS) $(TC_CPP)
+	$(NVCC) $(NVFLAGS) -Iinclude -shared $(TC_SRCS) $(TC_CPP) -o $@ -ldl 2> $(PKG)/ptxas.log || (cat $(PKG)/ptxas.log; false)
+
+clean:
+	rm -f graphgen/*.o graphgen/*.so oracle/*.so $(PKG)/*.so
+
+.PHONY: all clean
