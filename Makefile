@@ -5,7 +5,7 @@
 NVCC    ?= /usr/local/cuda/bin/nvcc
 CC      ?= gcc
 ARCH    := -gencode arch=compute_100a,code=sm_100a
-NVFLAGS := $(ARCH) -O3 -lineinfo -std=c++17 -Xcompiler -fPIC -Xcompiler -Wall \
+NVFLAGS := $(ARCH) -O3 -lineinfo -std=c++17 -Xcompiler -fPIC -Xcompiler -Wall -Xcompiler -ffp-contract=off \
            -Xptxas -v --expt-relaxed-constexpr
 CFLAGS  := -O2 -std=c11 -fPIC -Wall -Wextra -ffp-contract=off
 

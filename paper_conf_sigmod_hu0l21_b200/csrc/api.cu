@@ -1,0 +1,523 @@
+// api.cu — the C-ABI of include/tc.h: argument checks, the state machine, stage timing,
+// host/device pointer handling, exports, and the NCCL plumbing of tc_count_dist (a11).
+#include <dlfcn.h>
+
+#include <algorithm>
+#include <cstring>
+#include <map>
+#include <mutex>
+#include <new>
+#include <string>
+#include <vector>
+
+#include "internal.h"
+
+struct tc_graph : tc::Graph {
+  std::map<uint32_t, std::vector<uint32_t>> partitions;  // world -> bounds
+};
+
+namespace tc {
+
+int g_opt_profile = 1;
+static thread_local std::string t_err;
+
+void cuda_fail(cudaError_t e, const char *what, const char *file, int line) {
+  std::string msg = std::string(cudaGetErrorName(e)) + ": " + cudaGetErrorString(e) + " at " + what + " (" + file +
+                    ":" + std::to_string(line) + ")";
+  cudaGetLastError();
+  throw Error(e == cudaErrorMemoryAllocation ? ST_OOM : ST_CUDA, msg);
+}
+
+int num_sms() {
+  static int cached[64] = {0};
+  int dev = 0;
+  TC_CUDA(cudaGetDevice(&dev));
+  if (dev < 64 && cached[dev]) return cached[dev];
+  int sms = 0;
+  TC_CUDA(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+  if (dev < 64) cached[dev] = sms;
+  return sms;
+}
+
+template <class F>
+static tc_status guard(F &&f) {
+  try {
+    f();
+    return TC_OK;
+  } catch (const Error &e) {
+    t_err = e.what();
+    return (tc_status)e.status;
+  } catch (const std::bad_alloc &) {
+    t_err = "host allocation failed";
+    return TC_ERR_OOM;
+  } catch (const std::exception &e) {
+    t_err = e.what();
+    return TC_ERR_CUDA;
+  }
+}
+
+static void select_device(int device) {
+  int count = 0;
+  cudaError_t e = cudaGetDeviceCount(&count);
+  if (e != cudaSuccess || count == 0) {
+    cudaGetLastError();
+    throw Error(ST_CUDA, "no CUDA device available (libtc_b200 has no CPU fallback)");
+  }
+  TC_REQUIRE(device >= 0 && device < count, ST_INVALID, "device ordinal out of range");
+  TC_CUDA(cudaSetDevice(device));
+  static std::once_flag pool_once[64];
+  if (device < 64)
+    std::call_once(pool_once[device], [device] {
+      cudaMemPool_t pool;
+      if (cudaDeviceGetDefaultMemPool(&pool, device) == cudaSuccess) {
+        uint64_t thr = UINT64_MAX;  // keep freed blocks cached across graphs
+        cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+      }
+      cudaGetLastError();
+    });
+}
+
+static bool is_device_ptr(const void *p) {
+  if (!p) return false;
+  cudaPointerAttributes a;
+  if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
+}
+
+struct StageTimer {
+  cudaEvent_t a = nullptr, b = nullptr;
+  cudaStream_t s;
+  bool on;
+  explicit StageTimer(cudaStream_t st) : s(st), on(g_opt_profile != 0) {
+    if (!on) return;
+    TC_CUDA(cudaEventCreate(&a));
+    TC_CUDA(cudaEventCreate(&b));
+    TC_CUDA(cudaEventRecord(a, s));
+  }
+  double stop() {
+    if (!on) return 0.0;
+    TC_CUDA(cudaEventRecord(b, s));
+    TC_CUDA(cudaEventSynchronize(b));
+    float ms = 0;
+    TC_CUDA(cudaEventElapsedTime(&ms, a, b));
+    return ms;
+  }
+  ~StageTimer() {
+    if (a) cudaEventDestroy(a);
+    if (b) cudaEventDestroy(b);
+  }
+};
+
+static void copy_out(void *dst, const void *src, size_t bytes, cudaStream_t s) {
+  if (!bytes || !dst) return;
+  TC_REQUIRE(src != nullptr, ST_STATE, "requested data does not exist for this graph state");
+  TC_CUDA(cudaMemcpyAsync(dst, src, bytes, cudaMemcpyDefault, s));
+}
+
+static Graph &checked(tc_graph *g, GraphState need) {
+  TC_REQUIRE(g != nullptr, ST_INVALID, "graph is NULL");
+  TC_REQUIRE(g->state >= need, ST_STATE,
+             need == G_DIRECTED ? "call tc_direct first" : "graph not ready for this call");
+  TC_CUDA(cudaSetDevice(g->device));
+  return *g;
+}
+
+// ------------------------------------------------------------------ NCCL (dlopen)
+namespace nccl {
+typedef int Result;
+typedef struct Comm *Comm_t;
+struct UniqueId { char internal[128]; };
+enum { Uint64 = 5 };
+enum { Sum = 0 };
+struct Api {
+  void *h = nullptr;
+  Result (*GetUniqueId)(UniqueId *) = nullptr;
+  Result (*CommInitRank)(Comm_t *, int, UniqueId, int) = nullptr;
+  Result (*AllReduce)(const void *, void *, size_t, int, int, Comm_t, cudaStream_t) = nullptr;
+  Result (*CommDestroy)(Comm_t) = nullptr;
+  const char *(*GetErrorString)(Result) = nullptr;
+};
+static Api &api() {
+  static Api a;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    a.h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
+    if (!a.h) a.h = dlopen("libnccl.so", RTLD_NOW | RTLD_GLOBAL);
+    if (!a.h) return;
+    a.GetUniqueId = (Result(*)(UniqueId *))dlsym(a.h, "ncclGetUniqueId");
+    a.CommInitRank = (Result(*)(Comm_t *, int, UniqueId, int))dlsym(a.h, "ncclCommInitRank");
+    a.AllReduce = (Result(*)(const void *, void *, size_t, int, int, Comm_t, cudaStream_t))dlsym(a.h, "ncclAllReduce");
+    a.CommDestroy = (Result(*)(Comm_t))dlsym(a.h, "ncclCommDestroy");
+    a.GetErrorString = (const char *(*)(Result))dlsym(a.h, "ncclGetErrorString");
+  });
+  TC_REQUIRE(a.h && a.GetUniqueId && a.CommInitRank && a.AllReduce && a.CommDestroy, ST_NCCL,
+             "libnccl.so.2 not loadable");
+  return a;
+}
+static void check(Result r, const char *what) {
+  if (r != 0) {
+    const char *m = api().GetErrorString ? api().GetErrorString(r) : "?";
+    throw Error(ST_NCCL, std::string(what) + ": " + m);
+  }
+}
+}  // namespace nccl
+
+}  // namespace tc
+
+using namespace tc;
+
+extern "C" {
+
+const char *tc_last_error(void) { return t_err.c_str(); }
+const char *tc_version(void) { return "tc_b200 0.1 (sm_100a)"; }
+
+tc_status tc_set_option(const char *key, int64_t value) {
+  return guard([&] {
+    TC_REQUIRE(key != nullptr, ST_INVALID, "key is NULL");
+    std::string k(key);
+    if (k == "profile") g_opt_profile = value ? 1 : 0;
+    else if (k == "kernel_profile") g_opt_kernel_profile = value ? 1 : 0;
+    else if (k == "small_cap") {
+      TC_REQUIRE(value >= 32 && value <= 16384 && (value & (value - 1)) == 0, ST_INVALID,
+                 "small_cap must be a power of two in [32, 16384]");
+      g_opt_small_cap = (int)value;
+    } else throw Error(ST_INVALID, "unknown option " + k);
+  });
+}
+
+tc_status tc_graph_from_edges(const uint32_t *src, const uint32_t *dst, uint64_t num_edges, uint32_t num_vertices,
+                              int device, void *cuda_stream, tc_graph **out) {
+  return guard([&] {
+    TC_REQUIRE(out != nullptr, ST_INVALID, "out is NULL");
+    TC_REQUIRE(num_edges == 0 || (src && dst), ST_INVALID, "src/dst NULL with num_edges > 0");
+    select_device(device);
+    tc_graph *g = new tc_graph();
+    try {
+      g->device = device;
+      g->stream = (cudaStream_t)cuda_stream;
+      g->n = num_vertices;
+      StageTimer t(g->stream);
+      DevBuf<uint32_t> hs, hd;
+      const uint32_t *ds = src, *dd = dst;
+      if (num_edges && !is_device_ptr(src)) {
+        hs.alloc(num_edges, g->stream);
+        TC_CUDA(cudaMemcpyAsync(hs.get(), src, num_edges * 4, cudaMemcpyHostToDevice, g->stream));
+        ds = hs.get();
+      }
+      if (num_edges && !is_device_ptr(dst)) {
+        hd.alloc(num_edges, g->stream);
+        TC_CUDA(cudaMemcpyAsync(hd.get(), dst, num_edges * 4, cudaMemcpyHostToDevice, g->stream));
+        dd = hd.get();
+      }
+      build_graph(*g, ds, dd, num_edges);
+      hs.release();
+      hd.release();
+      g->ms_build = t.stop();
+      TC_CUDA(cudaStreamSynchronize(g->stream));
+    } catch (...) {
+      cudaStreamSynchronize(g->stream);
+      delete g;
+      throw;
+    }
+    *out = g;
+  });
+}
+
+tc_status tc_direct(tc_graph *gp, tc_direct_rule rule) {
+  return guard([&] {
+    Graph &g = checked(gp, G_BUILT);
+    TC_REQUIRE(rule >= TC_DIRECT_ID && rule <= TC_DIRECT_PAPER, ST_INVALID, "unknown directing rule");
+    StageTimer t(g.stream);
+    direct_graph(g, rule);
+    g.ms_direct = t.stop();
+    gp->partitions.clear();
+  });
+}
+
+static tc_aorder_params defaults_or(const tc_aorder_params *p) {
+  tc_aorder_params d;
+  d.lambda = 9.682;
+  d.alpha = 0.5;
+  d.beta = 0.5;
+  d.bw = nullptr;
+  d.bw_len = 0;
+  d.k = 32;
+  d.order = 0;
+  if (!p) return d;
+  TC_REQUIRE(p->k >= 1, ST_INVALID, "A-order: k must be >= 1");
+  TC_REQUIRE(p->bw == nullptr || p->bw_len >= 1, ST_INVALID, "A-order: bw_len must be >= 1");
+  TC_REQUIRE(p->order == 0 || p->order == 1, ST_INVALID, "A-order: order must be 0 or 1");
+  TC_REQUIRE(p->alpha > 0 && p->beta > 0, ST_INVALID, "A-order: alpha, beta must be > 0 (Eq.19-20)");
+  return *p;
+}
+
+tc_status tc_reorder(tc_graph *gp, tc_reorder_rule rule, const tc_aorder_params *p) {
+  return guard([&] {
+    Graph &g = checked(gp, G_DIRECTED);
+    TC_REQUIRE(rule >= TC_REORDER_NONE && rule <= TC_REORDER_PAPER, ST_INVALID, "unknown reorder rule");
+    tc_aorder_params prm = defaults_or(p);
+    StageTimer t(g.stream);
+    reorder_graph(g, rule, prm);
+    g.ms_reorder = t.stop();
+    gp->partitions.clear();
+  });
+}
+
+tc_status tc_set_schedule(tc_graph *gp, tc_schedule s) {
+  return guard([&] {
+    TC_REQUIRE(gp != nullptr, ST_INVALID, "graph is NULL");
+    TC_REQUIRE(s >= TC_SCHED_AUTO && s <= TC_SCHED_RANGE, ST_INVALID, "unknown schedule");
+    gp->schedule = s;
+  });
+}
+
+static void ensure_csr(Graph &g) {
+  if (!g.csr_ready) {
+    tc_aorder_params prm = defaults_or(nullptr);
+    reorder_graph(g, TC_REORDER_NONE, prm);
+  }
+}
+
+static uint64_t do_count(tc_graph *gp, uint32_t ub, uint32_t ue, uint64_t *per_vertex, void *comm, bool reduce) {
+  Graph &g = *gp;
+  StageTimer t(g.stream);
+  ensure_csr(g);
+  DevBuf<uint64_t> tnew;
+  if (per_vertex) {
+    tnew.alloc(g.n ? g.n : 1, g.stream);
+    TC_CUDA(cudaMemsetAsync(tnew.get(), 0, tnew.bytes(), g.stream));
+  }
+  float kms = 0;
+  uint64_t launches = 0;
+  uint64_t T = count_graph(g, ub, ue, per_vertex ? tnew.get() : nullptr, g_opt_profile ? &kms : nullptr, &launches);
+  if (reduce) {
+    nccl::Api &a = nccl::api();
+    DevBuf<uint64_t> dT;
+    dT.alloc(1, g.stream);
+    TC_CUDA(cudaMemcpyAsync(dT.get(), &T, 8, cudaMemcpyHostToDevice, g.stream));
+    nccl::check(a.AllReduce(dT.get(), dT.get(), 1, nccl::Uint64, nccl::Sum, (nccl::Comm_t)comm, g.stream),
+                "ncclAllReduce(T)");
+    if (per_vertex && g.n)
+      nccl::check(a.AllReduce(tnew.get(), tnew.get(), g.n, nccl::Uint64, nccl::Sum, (nccl::Comm_t)comm, g.stream),
+                  "ncclAllReduce(per_vertex)");
+    TC_CUDA(cudaMemcpyAsync(&T, dT.get(), 8, cudaMemcpyDeviceToHost, g.stream));
+    TC_CUDA(cudaStreamSynchronize(g.stream));
+  }
+  if (per_vertex && g.n) {
+    if (is_device_ptr(per_vertex)) {
+      gather_per_vertex(g, tnew.get(), per_vertex);
+    } else {
+      DevBuf<uint64_t> tmp;
+      tmp.alloc(g.n, g.stream);
+      gather_per_vertex(g, tnew.get(), tmp.get());
+      TC_CUDA(cudaMemcpyAsync(per_vertex, tmp.get(), 8ull * g.n, cudaMemcpyDeviceToHost, g.stream));
+      TC_CUDA(cudaStreamSynchronize(g.stream));
+    }
+  }
+  TC_CUDA(cudaStreamSynchronize(g.stream));
+  g.ms_count = t.stop();
+  g.ms_count_kernel = kms;
+  g.count_launches = launches;
+  g.triangles = T;
+  return T;
+}
+
+tc_status tc_count(tc_graph *gp, uint64_t *triangles, uint64_t *per_vertex) {
+  return guard([&] {
+    checked(gp, G_DIRECTED);
+    TC_REQUIRE(triangles != nullptr, ST_INVALID, "triangles is NULL");
+    uint64_t T = do_count(gp, 0, gp->n, per_vertex, nullptr, false);
+    *triangles = T;
+  });
+}
+
+tc_status tc_count_range(tc_graph *gp, uint32_t u_begin, uint32_t u_end, uint64_t *triangles,
+                         uint64_t *per_vertex) {
+  return guard([&] {
+    checked(gp, G_DIRECTED);
+    TC_REQUIRE(triangles != nullptr, ST_INVALID, "triangles is NULL");
+    TC_REQUIRE(u_begin <= u_end && u_end <= gp->n, ST_INVALID, "bad vertex range");
+    uint64_t T = do_count(gp, u_begin, u_end, per_vertex, nullptr, false);
+    *triangles = T;
+  });
+}
+
+tc_status tc_partition(tc_graph *gp, uint32_t world, uint32_t *bounds) {
+  return guard([&] {
+    Graph &g = checked(gp, G_DIRECTED);
+    TC_REQUIRE(world >= 1 && bounds != nullptr, ST_INVALID, "world >= 1 and bounds required");
+    ensure_csr(g);
+    auto it = gp->partitions.find(world);
+    if (it == gp->partitions.end()) {
+      std::vector<uint32_t> b(world + 1);
+      partition_graph(g, world, b.data());
+      // RANGE schedule after A-order: snap to bucket starts so buckets stay whole
+      if (!g.h_bucket_off.empty()) {
+        const auto &hb = g.h_bucket_off;
+        for (uint32_t r = 1; r < world; ++r) {
+          auto pos = std::lower_bound(hb.begin(), hb.end(), b[r]);
+          if (pos != hb.end()) b[r] = *pos;
+          else b[r] = g.n;
+          b[r] = std::max(b[r], b[r - 1]);
+        }
+      }
+      it = gp->partitions.emplace(world, std::move(b)).first;
+    }
+    std::memcpy(bounds, it->second.data(), sizeof(uint32_t) * (world + 1));
+  });
+}
+
+tc_status tc_nccl_get_unique_id(void *unique_id) {
+  return guard([&] {
+    TC_REQUIRE(unique_id != nullptr, ST_INVALID, "unique_id is NULL");
+    nccl::UniqueId id;
+    nccl::check(nccl::api().GetUniqueId(&id), "ncclGetUniqueId");
+    std::memcpy(unique_id, &id, sizeof(id));
+  });
+}
+
+tc_status tc_nccl_comm_init(const void *unique_id, int rank, int world, int device, void **comm) {
+  return guard([&] {
+    TC_REQUIRE(unique_id && comm && world >= 1 && rank >= 0 && rank < world, ST_INVALID, "bad NCCL init args");
+    select_device(device);
+    nccl::UniqueId id;
+    std::memcpy(&id, unique_id, sizeof(id));
+    nccl::Comm_t c = nullptr;
+    nccl::check(nccl::api().CommInitRank(&c, world, id, rank), "ncclCommInitRank");
+    *comm = c;
+  });
+}
+
+tc_status tc_nccl_comm_destroy(void *comm) {
+  return guard([&] {
+    if (comm) nccl::check(nccl::api().CommDestroy((nccl::Comm_t)comm), "ncclCommDestroy");
+  });
+}
+
+tc_status tc_count_dist(tc_graph *gp, void *comm, int rank, int world, uint64_t *triangles, uint64_t *per_vertex) {
+  return guard([&] {
+    checked(gp, G_DIRECTED);
+    TC_REQUIRE(triangles != nullptr && comm != nullptr, ST_INVALID, "triangles/comm NULL");
+    TC_REQUIRE(world >= 1 && rank >= 0 && rank < world, ST_INVALID, "bad rank/world");
+    std::vector<uint32_t> b(world + 1);
+    tc_status st = tc_partition(gp, (uint32_t)world, b.data());
+    if (st != TC_OK) throw Error(st, t_err);
+    uint64_t T = do_count(gp, b[rank], b[rank + 1], per_vertex, comm, true);
+    *triangles = T;
+  });
+}
+
+tc_status tc_analyze(tc_graph *gp) {
+  return guard([&] {
+    Graph &g = checked(gp, G_DIRECTED);
+    ensure_csr(g);
+    analyze_graph(g);
+  });
+}
+
+tc_status tc_get_stats(const tc_graph *gp, tc_stats_t *o) {
+  return guard([&] {
+    TC_REQUIRE(gp && o, ST_INVALID, "NULL argument");
+    const Graph &g = *gp;
+    std::memset(o, 0, sizeof(*o));
+    o->n = g.n;
+    o->m = g.m;
+    o->samples = g.samples;
+    o->max_degree = g.max_degree;
+    o->max_outdeg = g.max_outdeg;
+    o->eq1_lo = g.eq1_lo;
+    o->eq1_hi = g.eq1_hi;
+    o->eq3 = g.eq3;
+    o->levels = g.levels;
+    o->subrounds = g.subrounds;
+    o->nbuckets = g.h_bucket_off.empty() ? 0 : (uint32_t)g.h_bucket_off.size() - 1;
+    o->direct_rule = (uint32_t)g.direct_rule;
+    o->reorder_rule = (uint32_t)g.reorder_rule;
+    o->schedule = (uint32_t)g.schedule;
+    o->triangles = g.triangles;
+    o->wedges = g.wedges;
+    o->alg_bytes = g.alg_bytes;
+    o->ms_build = g.ms_build;
+    o->ms_direct = g.ms_direct;
+    o->ms_reorder = g.ms_reorder;
+    o->ms_count = g.ms_count;
+    o->ms_count_kernel = g.ms_count_kernel;
+    o->count_launches = g.count_launches;
+  });
+}
+
+tc_status tc_export(tc_graph *gp, uint64_t *offs, uint32_t *col, uint32_t *perm) {
+  return guard([&] {
+    Graph &g = checked(gp, G_DIRECTED);
+    ensure_csr(g);
+    copy_out(offs, g.offs.get(), 8ull * (g.n + 1ull), g.stream);
+    copy_out(col, g.col.get(), 4ull * g.m, g.stream);
+    if (perm && g.n) {
+      if (g.identity_perm) {
+        std::vector<uint32_t> id(g.n);
+        for (uint32_t i = 0; i < g.n; ++i) id[i] = i;
+        copy_out(perm, id.data(), 4ull * g.n, g.stream);
+        TC_CUDA(cudaStreamSynchronize(g.stream));
+      } else {
+        copy_out(perm, g.perm.get(), 4ull * g.n, g.stream);
+      }
+    }
+    TC_CUDA(cudaStreamSynchronize(g.stream));
+  });
+}
+
+__global__ void unpack_edges_kernel(const uint64_t *in, uint64_t m, int bits, uint64_t *out) {
+  uint64_t mask = (1ull << bits) - 1;
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < m; i += (uint64_t)gridDim.x * blockDim.x)
+    out[i] = ((in[i] >> bits) << 32) | (in[i] & mask);
+}
+
+tc_status tc_export_graph(tc_graph *gp, uint64_t *edges, uint32_t *degree) {
+  return guard([&] {
+    Graph &g = checked(gp, G_BUILT);
+    if (edges && g.m) {
+      DevBuf<uint64_t> tmp;
+      tmp.alloc(g.m, g.stream);
+      unpack_edges_kernel<<<grid_for(g.m, 256), 256, 0, g.stream>>>(g.edges.get(), g.m, g.bits, tmp.get());
+      TC_LAUNCH_CHECK();
+      copy_out(edges, tmp.get(), 8ull * g.m, g.stream);
+      TC_CUDA(cudaStreamSynchronize(g.stream));
+    }
+    copy_out(degree, g.deg.get(), 4ull * g.n, g.stream);
+    TC_CUDA(cudaStreamSynchronize(g.stream));
+  });
+}
+
+tc_status tc_export_direct(tc_graph *gp, uint32_t *outdeg, uint32_t *sub, uint32_t *dsnap) {
+  return guard([&] {
+    Graph &g = checked(gp, G_DIRECTED);
+    TC_REQUIRE(!(sub || dsnap) || g.direct_rule == TC_DIRECT_PAPER, ST_STATE, "sub/dsnap exist only for PAPER");
+    copy_out(outdeg, g.od.get(), 4ull * g.n, g.stream);
+    copy_out(sub, g.sub.get(), 4ull * g.n, g.stream);
+    copy_out(dsnap, g.dsnap.get(), 4ull * g.n, g.stream);
+    TC_CUDA(cudaStreamSynchronize(g.stream));
+  });
+}
+
+tc_status tc_export_buckets(tc_graph *gp, uint32_t *bucket_off) {
+  return guard([&] {
+    Graph &g = checked(gp, G_DIRECTED);
+    TC_REQUIRE(!g.h_bucket_off.empty(), ST_STATE, "no A-order buckets (tc_reorder PAPER first)");
+    copy_out(bucket_off, g.h_bucket_off.data(), 4ull * g.h_bucket_off.size(), g.stream);
+    TC_CUDA(cudaStreamSynchronize(g.stream));
+  });
+}
+
+void tc_graph_free(tc_graph *gp) {
+  if (!gp) return;
+  cudaSetDevice(gp->device);
+  cudaStream_t s = gp->stream;
+  delete gp;  // DevBufs free stream-ordered
+  cudaStreamSynchronize(s);
+  cudaGetLastError();
+}
+
+}  // extern "C"

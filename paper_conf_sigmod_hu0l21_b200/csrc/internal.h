@@ -1,0 +1,78 @@
+// internal.h — the tc_graph object and the host-side stage functions of libtc_b200.
+#pragma once
+#include <stdint.h>
+
+#include <vector>
+
+#include "../../include/tc.h"
+#include "common.cuh"
+
+namespace tc {
+
+enum GraphState { G_BUILT = 0, G_DIRECTED = 1, G_ORDERED = 2 };
+
+struct StageTimer;  // CUDA-event stage timing (api.cu)
+
+struct Graph {
+  int device = 0;
+  cudaStream_t stream = nullptr;
+  uint32_t n = 0;
+  uint64_t m = 0, samples = 0;
+  int bits = 1;  // bits(n-1): packed key (hi << bits) | lo
+  GraphState state = G_BUILT;
+
+  // a1-a3: simple undirected graph
+  DevBuf<uint64_t> edges;  // m packed keys (u << bits) | v, u < v, ascending
+  DevBuf<uint32_t> deg;    // d(v)
+  uint32_t max_degree = 0;
+
+  // a4-a5: directing
+  int direct_rule = -1;
+  DevBuf<uint64_t> prim;   // orientation key: u->v iff (prim[u], u) < (prim[v], v)
+  DevBuf<uint32_t> od;     // out-degree d~ (original ids)
+  DevBuf<uint32_t> sub, dsnap;  // A-direction internals (PAPER only)
+  uint32_t levels = 0, subrounds = 0, max_outdeg = 0;
+  uint64_t eq1_lo = 0, eq1_hi = 0;
+
+  // a6-a7: ordering + oriented CSR (final labels)
+  int reorder_rule = -1;
+  bool identity_perm = true;
+  DevBuf<uint32_t> perm;          // perm[old] = new (empty if identity)
+  std::vector<uint32_t> h_bucket_off;  // A-order buckets (host)
+  DevBuf<uint32_t> bucket_off;    // A-order buckets (device)
+  int64_t eq3 = -1;
+  DevBuf<uint64_t> offs;          // n+1
+  DevBuf<uint32_t> col;           // m (+ 8 padding words)
+  bool csr_ready = false;
+
+  // a8 schedule
+  int schedule = TC_SCHED_AUTO;
+
+  // results / stats
+  uint64_t triangles = 0, wedges = 0, alg_bytes = 0;
+  double ms_build = 0, ms_direct = 0, ms_reorder = 0, ms_count = 0, ms_count_kernel = 0;
+  uint64_t count_launches = 0;
+};
+
+// build.cu
+void build_graph(Graph &g, const uint32_t *d_src, const uint32_t *d_dst, uint64_t M);
+// direct.cu
+void direct_graph(Graph &g, int rule);
+// reorder.cu
+void reorder_graph(Graph &g, int rule, const tc_aorder_params &p);
+void build_oriented_csr(Graph &g);
+// aorder.cpp (host, Algorithm 2)
+void aorder_host(const std::vector<uint32_t> &od, const tc_aorder_params &p, std::vector<uint32_t> &perm,
+                 std::vector<uint32_t> &bucket_off, int64_t &eq3);
+// count.cu
+uint64_t count_graph(Graph &g, uint32_t u_begin, uint32_t u_end, uint64_t *d_tv /*new labels or null*/,
+                     float *kernel_ms, uint64_t *launches);
+void gather_per_vertex(Graph &g, const uint64_t *d_tnew, uint64_t *d_out);
+void partition_graph(Graph &g, uint32_t world, uint32_t *bounds);
+void analyze_graph(Graph &g);
+
+// options (api.cu)
+extern int g_opt_profile;
+extern int g_opt_small_cap;
+
+}  // namespace tc

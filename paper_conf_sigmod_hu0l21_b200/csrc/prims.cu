@@ -1,0 +1,289 @@
+// prims.cu — one-sweep LSD radix sort, look-back scan and unique-select for sm_100a.
+//
+// All three are single-pass over their input per digit/scan using decoupled look-back
+// (tiles obtain their index from an atomic counter, publish an aggregate, then the
+// inclusive prefix), so each radix pass reads and writes the keys exactly once
+// (16 B per key per pass of HBM traffic), plus one up-front read for all digit
+// histograms.  Digits are 8 bits; only the significant bits are sorted (the CSR
+// build packs (u, v) into 2*ceil(log2 n) bits).
+#include "prims.cuh"
+
+namespace tc {
+
+namespace {
+
+constexpr int T_THREADS = 256;
+constexpr int T_ITEMS = 16;
+constexpr int T_TILE = T_THREADS * T_ITEMS;  // 4096
+constexpr int T_WARPS = T_THREADS / 32;
+constexpr int MAX_PASSES = 8;
+
+// ------------------------------------------------------------------ scan
+template <typename TI>
+__global__ __launch_bounds__(T_THREADS) void scan_kernel(const TI *__restrict__ in,
+                                                             uint64_t *__restrict__ out, uint64_t n,
+                                                             uint64_t *status, uint32_t *tile_ctr) {
+  __shared__ uint64_t s_warp[8];
+  __shared__ uint64_t s_total;
+  __shared__ uint32_t s_tile;
+  __shared__ uint64_t s_excl;
+  if (threadIdx.x == 0) s_tile = atomicAdd(tile_ctr, 1u);
+  __syncthreads();
+  uint64_t tile = s_tile;
+  uint64_t base = tile * T_TILE + (uint64_t)threadIdx.x * T_ITEMS;
+  uint64_t v[T_ITEMS];
+  uint64_t sum = 0;
+#pragma unroll
+  for (int i = 0; i < T_ITEMS; ++i) {
+    uint64_t idx = base + i;
+    v[i] = idx < n ? (uint64_t)in[idx] : 0ull;
+    sum += v[i];
+  }
+  uint64_t excl_t = block256_exclusive_scan<uint64_t>(sum, s_warp, &s_total);
+  if (threadIdx.x == 0) s_excl = lookback_exclusive(status, tile, 1, s_total);
+  __syncthreads();
+  uint64_t run = s_excl + excl_t;
+#pragma unroll
+  for (int i = 0; i < T_ITEMS; ++i) {
+    uint64_t idx = base + i;
+    if (idx <= n) out[idx] = run;  // out[n] = total
+    run += v[i];
+  }
+}
+
+// ------------------------------------------------------------------ unique
+__global__ __launch_bounds__(T_THREADS) void unique_kernel(const uint64_t *__restrict__ in,
+                                                           uint64_t *__restrict__ out, uint64_t n,
+                                                           uint64_t *status, uint32_t *tile_ctr,
+                                                           uint64_t ntiles, uint64_t *d_count) {
+  __shared__ uint64_t s_warp[8];
+  __shared__ uint64_t s_total;
+  __shared__ uint32_t s_tile;
+  __shared__ uint64_t s_excl;
+  if (threadIdx.x == 0) s_tile = atomicAdd(tile_ctr, 1u);
+  __syncthreads();
+  uint64_t tile = s_tile;
+  uint64_t base = tile * T_TILE + (uint64_t)threadIdx.x * T_ITEMS;
+  uint64_t k[T_ITEMS];
+  uint32_t flags = 0;
+  uint64_t prev = (base > 0 && base <= n) ? in[base - 1] : 0;
+#pragma unroll
+  for (int i = 0; i < T_ITEMS; ++i) {
+    uint64_t idx = base + i;
+    k[i] = idx < n ? in[idx] : 0;
+    bool head = idx < n && (idx == 0 || k[i] != prev);
+    flags |= (uint32_t)head << i;
+    prev = k[i];
+  }
+  uint64_t cnt = __popc(flags);
+  uint64_t excl_t = block256_exclusive_scan<uint64_t>(cnt, s_warp, &s_total);
+  if (threadIdx.x == 0) {
+    s_excl = lookback_exclusive(status, tile, 1, s_total);
+    if (tile == ntiles - 1) *d_count = s_excl + s_total;
+  }
+  __syncthreads();
+  uint64_t pos = s_excl + excl_t;
+#pragma unroll
+  for (int i = 0; i < T_ITEMS; ++i)
+    if (flags >> i & 1u) out[pos++] = k[i];
+}
+
+// ------------------------------------------------------------------ radix sort
+// Up-front digit histograms for every pass; per-warp private smem counters.
+__global__ __launch_bounds__(T_THREADS) void rs_hist_kernel(const uint64_t *__restrict__ keys,
+                                                            uint64_t n, int begin_bit, int passes,
+                                                            unsigned long long *ghist) {
+  extern __shared__ uint32_t s_h[];  // [T_WARPS/2][passes][256]
+  const int groups = T_WARPS / 2;
+  for (int i = threadIdx.x; i < groups * passes * 256; i += T_THREADS) s_h[i] = 0;
+  __syncthreads();
+  uint32_t *mine = s_h + (warp_id() / 2) * passes * 256;
+  uint64_t stride = (uint64_t)gridDim.x * T_THREADS;
+  for (uint64_t i = (uint64_t)blockIdx.x * T_THREADS + threadIdx.x; i < n; i += stride) {
+    uint64_t k = keys[i];
+    for (int p = 0; p < passes; ++p) atomicAdd(&mine[p * 256 + ((k >> (begin_bit + 8 * p)) & 255u)], 1u);
+  }
+  __syncthreads();
+  for (int i = threadIdx.x; i < passes * 256; i += T_THREADS) {
+    uint32_t c = 0;
+    for (int g = 0; g < groups; ++g) c += s_h[g * passes * 256 + i];
+    if (c) atomicAdd(&ghist[i], (unsigned long long)c);
+  }
+}
+
+__global__ void rs_hist_scan_kernel(unsigned long long *ghist, int passes) {
+  // one block of 256 threads: exclusive scan of each pass' 256 bins, in place
+  __shared__ uint64_t s_warp[8];
+  __shared__ uint64_t s_total;
+  for (int p = 0; p < passes; ++p) {
+    uint64_t v = ghist[p * 256 + threadIdx.x];
+    uint64_t e = block256_exclusive_scan<uint64_t>(v, s_warp, &s_total);
+    __syncthreads();
+    ghist[p * 256 + threadIdx.x] = e;
+    __syncthreads();
+  }
+}
+
+__global__ __launch_bounds__(T_THREADS) void rs_pass_kernel(const uint64_t *__restrict__ in,
+                                                            uint64_t *__restrict__ out, uint64_t n,
+                                                            int shift,
+                                                            const unsigned long long *__restrict__ goff,
+                                                            uint64_t *status, uint32_t *tile_ctr) {
+  __shared__ uint64_t s_keys[T_TILE];
+  __shared__ uint32_t s_whist[T_WARPS][256];
+  __shared__ uint32_t s_lstart[256];
+  __shared__ uint64_t s_gbase[256];
+  __shared__ uint32_t s_warp32[8];
+  __shared__ uint32_t s_total32;
+  __shared__ uint32_t s_tile;
+  const unsigned w = warp_id(), l = lane_id(), t = threadIdx.x;
+  if (t == 0) s_tile = atomicAdd(tile_ctr, 1u);
+#pragma unroll
+  for (int i = 0; i < T_WARPS; ++i) s_whist[i][t] = 0;
+  __syncthreads();
+  const uint64_t tile = s_tile;
+  const uint64_t base = tile * T_TILE;
+
+  uint64_t k[T_ITEMS];
+  uint32_t d[T_ITEMS];
+  uint32_t r[T_ITEMS];
+#pragma unroll
+  for (int i = 0; i < T_ITEMS; ++i) {
+    uint64_t idx = base + w * (32 * T_ITEMS) + i * 32 + l;  // warp-striped: stable order
+    bool valid = idx < n;
+    k[i] = valid ? in[idx] : ~0ull;
+    d[i] = valid ? (uint32_t)((k[i] >> shift) & 255u) : 256u;
+  }
+  const unsigned lt_mask = (1u << l) - 1u;
+#pragma unroll
+  for (int i = 0; i < T_ITEMS; ++i) {
+    unsigned peers = __match_any_sync(0xffffffffu, d[i]);
+    unsigned lead = __ffs(peers) - 1;
+    uint32_t cur = d[i] < 256u ? s_whist[w][d[i]] : 0u;
+    r[i] = cur + __popc(peers & lt_mask);
+    __syncwarp();
+    if (l == lead && d[i] < 256u) s_whist[w][d[i]] = cur + __popc(peers);
+    __syncwarp();
+  }
+  __syncthreads();
+  // digit t: exclusive prefix over warps, tile count
+  uint32_t run = 0;
+#pragma unroll
+  for (int ww = 0; ww < T_WARPS; ++ww) {
+    uint32_t c = s_whist[ww][t];
+    s_whist[ww][t] = run;
+    run += c;
+  }
+  uint32_t lstart = block256_exclusive_scan<uint32_t>(run, s_warp32, &s_total32);
+  s_lstart[t] = lstart;
+  // look-back for digit t (status laid out [tile][256])
+  {
+    uint64_t *st = status + t;
+    uint64_t e = 0;
+    if (tile == 0) {
+      st_relaxed_u64(st, LB_INC | run);
+    } else {
+      st_relaxed_u64(st + tile * 256, LB_AGG | run);
+      int64_t j = (int64_t)tile - 1;
+      while (true) {
+        uint64_t sv = ld_relaxed_u64(st + (uint64_t)j * 256);
+        uint64_t f = sv & ~LB_VAL;
+        if (f == 0) continue;
+        e += sv & LB_VAL;
+        if (f == LB_INC) break;
+        --j;
+      }
+      st_relaxed_u64(st + tile * 256, LB_INC | (e + run));
+    }
+    s_gbase[t] = goff[t] + e;
+  }
+  __syncthreads();
+#pragma unroll
+  for (int i = 0; i < T_ITEMS; ++i)
+    if (d[i] < 256u) s_keys[s_lstart[d[i]] + s_whist[w][d[i]] + r[i]] = k[i];
+  __syncthreads();
+  uint64_t valid_count = n - base < (uint64_t)T_TILE ? n - base : (uint64_t)T_TILE;
+  for (uint32_t j = t; j < valid_count; j += T_THREADS) {
+    uint64_t key = s_keys[j];
+    uint32_t dd = (uint32_t)((key >> shift) & 255u);
+    out[s_gbase[dd] + j - s_lstart[dd]] = key;
+  }
+}
+
+}  // namespace
+
+template <typename TI>
+static void scan_impl(const TI *in, uint64_t *out, uint64_t n, cudaStream_t s) {
+  uint64_t ntiles = (n + 1 + T_TILE - 1) / T_TILE;  // +1: the total at out[n]
+  DevBuf<uint64_t> scratch;
+  scratch.alloc(ntiles + 1, s);
+  TC_CUDA(cudaMemsetAsync(scratch.get(), 0, scratch.bytes(), s));
+  ProfScope prof("scan", s, (double)n * sizeof(TI) + 8.0 * (n + 1));
+  scan_kernel<TI><<<(unsigned)ntiles, T_THREADS, 0, s>>>(in, out, n, scratch.get() + 1,
+                                                         (uint32_t *)scratch.get());
+  TC_LAUNCH_CHECK();
+}
+
+void scan_u32_to_u64(const uint32_t *in, uint64_t *out, uint64_t n, cudaStream_t s) {
+  scan_impl<uint32_t>(in, out, n, s);
+}
+void scan_u64(const uint64_t *in, uint64_t *out, uint64_t n, cudaStream_t s) {
+  scan_impl<uint64_t>(in, out, n, s);
+}
+
+void unique_sorted_u64(const uint64_t *in, uint64_t *out, uint64_t n, uint64_t *d_count,
+                       cudaStream_t s) {
+  if (n == 0) {
+    TC_CUDA(cudaMemsetAsync(d_count, 0, sizeof(uint64_t), s));
+    return;
+  }
+  uint64_t ntiles = (n + T_TILE - 1) / T_TILE;
+  DevBuf<uint64_t> scratch;
+  scratch.alloc(ntiles + 1, s);
+  TC_CUDA(cudaMemsetAsync(scratch.get(), 0, scratch.bytes(), s));
+  ProfScope prof("unique", s, 8.0 * n);
+  unique_kernel<<<(unsigned)ntiles, T_THREADS, 0, s>>>(in, out, n, scratch.get() + 1,
+                                                       (uint32_t *)scratch.get(), ntiles, d_count);
+  TC_LAUNCH_CHECK();
+}
+
+uint64_t *radix_sort_u64(uint64_t *keys, uint64_t *tmp, uint64_t n, int begin_bit, int end_bit,
+                         cudaStream_t s) {
+  if (n <= 1 || end_bit <= begin_bit) return keys;
+  int passes = (end_bit - begin_bit + 7) / 8;
+  TC_REQUIRE(passes <= MAX_PASSES, ST_INVALID, "radix sort: too many bits");
+  uint64_t ntiles = (n + T_TILE - 1) / T_TILE;
+  DevBuf<unsigned long long> hist;
+  hist.alloc((size_t)passes * 256, s);
+  TC_CUDA(cudaMemsetAsync(hist.get(), 0, hist.bytes(), s));
+  size_t hsm = (size_t)(T_WARPS / 2) * passes * 256 * sizeof(uint32_t);
+  static bool attr_set = false;
+  if (!attr_set) {
+    TC_CUDA(cudaFuncSetAttribute(rs_hist_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 (int)((T_WARPS / 2) * MAX_PASSES * 256 * sizeof(uint32_t))));
+    attr_set = true;
+  }
+  {
+    ProfScope prof("radix_hist", s, 8.0 * n);
+    rs_hist_kernel<<<grid_for(n, T_THREADS, 4), T_THREADS, hsm, s>>>(keys, n, begin_bit, passes,
+                                                                     hist.get());
+    TC_LAUNCH_CHECK();
+  }
+  rs_hist_scan_kernel<<<1, 256, 0, s>>>(hist.get(), passes);
+  TC_LAUNCH_CHECK();
+  DevBuf<uint64_t> scratch;  // [tile counter][status ntiles*256]
+  scratch.alloc(1 + ntiles * 256, s);
+  uint64_t *src = keys, *dst = tmp;
+  for (int p = 0; p < passes; ++p) {
+    TC_CUDA(cudaMemsetAsync(scratch.get(), 0, scratch.bytes(), s));
+    ProfScope prof("radix_pass", s, 16.0 * n);
+    rs_pass_kernel<<<(unsigned)ntiles, T_THREADS, 0, s>>>(src, dst, n, begin_bit + 8 * p,
+                                                          hist.get() + p * 256, scratch.get() + 1,
+                                                          (uint32_t *)scratch.get());
+    TC_LAUNCH_CHECK();
+    std::swap(src, dst);
+  }
+  return src;
+}
+
+}  // namespace tc

@@ -1,0 +1,147 @@
+// reorder.cu — steps a6-a7: vertex ordering and the oriented CSR in the new labels.
+//
+//   NONE    identity ("Original")
+//   DEGREE  D-order: descending out-degree d~, ties by id (Q14) — one radix sort of
+//           ((max d~ - d~(v)) << bits(n)) | v
+//   PAPER   A-order (Algorithm 2) on the host (aorder.cpp), perm and bucket offsets uploaded
+// Oriented CSR: each undirected edge {u,v} becomes (π(src), π(dst)) with src the earlier
+// endpoint in the directing order; keys (π(src) << b) | π(dst) are radix-sorted,
+// giving ascending lists N+(x) (the layout binary search needs); offsets are the
+// exclusive scan of d~ in the new labels.
+#include <vector>
+
+#include "internal.h"
+#include "prims.cuh"
+
+namespace tc {
+namespace {
+
+__global__ void dorder_keys_kernel(const uint32_t *__restrict__ od, uint32_t n, uint32_t maxod, int bn,
+                                   uint64_t *__restrict__ keys) {
+  for (uint64_t v = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (uint64_t)gridDim.x * blockDim.x)
+    keys[v] = ((uint64_t)(maxod - od[v]) << bn) | v;
+}
+
+__global__ void perm_from_sorted_kernel(const uint64_t *__restrict__ keys, uint32_t n, uint64_t mask,
+                                        uint32_t *__restrict__ perm) {
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
+    perm[keys[i] & mask] = (uint32_t)i;
+}
+
+template <bool IDENT>
+__global__ void orient_keys_kernel(const uint64_t *__restrict__ edges, uint64_t m, int bits,
+                                   const uint64_t *__restrict__ prim, const uint32_t *__restrict__ perm,
+                                   uint64_t *__restrict__ keys) {
+  uint64_t mask = (1ull << bits) - 1;
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < m; i += (uint64_t)gridDim.x * blockDim.x) {
+    uint64_t k = edges[i];
+    uint32_t u = (uint32_t)(k >> bits), v = (uint32_t)(k & mask);  // u < v
+    bool ufirst = prim[u] <= prim[v];
+    uint32_t s = ufirst ? u : v, t = ufirst ? v : u;
+    if (!IDENT) { s = perm[s]; t = perm[t]; }
+    keys[i] = ((uint64_t)s << bits) | t;
+  }
+}
+
+__global__ void scatter_od_kernel(const uint32_t *__restrict__ od, const uint32_t *__restrict__ perm, uint32_t n,
+                                  uint32_t *__restrict__ od_new) {
+  for (uint64_t v = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (uint64_t)gridDim.x * blockDim.x)
+    od_new[perm[v]] = od[v];
+}
+
+__global__ void extract_col_kernel(const uint64_t *__restrict__ keys, uint64_t m, uint64_t mask,
+                                   uint32_t *__restrict__ col) {
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < m; i += (uint64_t)gridDim.x * blockDim.x)
+    col[i] = (uint32_t)(keys[i] & mask);
+}
+
+}  // namespace
+
+uint32_t device_max_u32(const uint32_t *a, uint64_t n, cudaStream_t s);
+
+void build_oriented_csr(Graph &g) {
+  cudaStream_t s = g.stream;
+  const uint32_t n = g.n;
+  const uint64_t m = g.m;
+  const int b = g.bits;
+  const bool ident = g.identity_perm;
+  DevBuf<uint64_t> keys, tmp;
+  keys.alloc(m ? m : 1, s);
+  if (m) {
+    ProfScope prof("orient_keys", s, 24.0 * m);
+    if (ident)
+      orient_keys_kernel<true><<<grid_for(m, 256), 256, 0, s>>>(g.edges.get(), m, b, g.prim.get(), nullptr, keys.get());
+    else
+      orient_keys_kernel<false><<<grid_for(m, 256), 256, 0, s>>>(g.edges.get(), m, b, g.prim.get(), g.perm.get(),
+                                                                  keys.get());
+    TC_LAUNCH_CHECK();
+  }
+  uint64_t *sorted = keys.get();
+  if (!(ident && g.direct_rule == TC_DIRECT_ID)) {  // ID order + identity: already sorted
+    tmp.alloc(m ? m : 1, s);
+    sorted = radix_sort_u64(keys.get(), tmp.get(), m, 0, 2 * b, s);
+  }
+  // offsets from d~ in the new labels
+  g.offs.alloc((uint64_t)n + 1, s);
+  if (ident) {
+    scan_u32_to_u64(g.od.get(), g.offs.get(), n, s);
+  } else {
+    DevBuf<uint32_t> odn;
+    odn.alloc(n ? n : 1, s);
+    if (n) scatter_od_kernel<<<grid_for(n, 256), 256, 0, s>>>(g.od.get(), g.perm.get(), n, odn.get());
+    TC_LAUNCH_CHECK();
+    scan_u32_to_u64(odn.get(), g.offs.get(), n, s);
+  }
+  g.col.alloc(m + 32, s);  // tail padding: vectorised loads may over-read by < 16 B
+  TC_CUDA(cudaMemsetAsync(g.col.get() + m, 0xff, 32 * sizeof(uint32_t), s));
+  if (m) {
+    ProfScope prof("extract_col", s, 12.0 * m);
+    extract_col_kernel<<<grid_for(m, 256), 256, 0, s>>>(sorted, m, (1ull << b) - 1, g.col.get());
+    TC_LAUNCH_CHECK();
+  }
+  g.csr_ready = true;
+}
+
+void reorder_graph(Graph &g, int rule, const tc_aorder_params &p) {
+  cudaStream_t s = g.stream;
+  const uint32_t n = g.n;
+  g.perm.release();
+  g.bucket_off.release();
+  g.h_bucket_off.clear();
+  g.eq3 = -1;
+  g.identity_perm = true;
+  if (rule == TC_REORDER_DEGREE && n > 1) {
+    int bn = bits_for(n - 1);
+    uint32_t maxod = g.max_outdeg;
+    int kb = bits_for(maxod) + bn;
+    DevBuf<uint64_t> keys, tmp;
+    keys.alloc(n, s);
+    tmp.alloc(n, s);
+    dorder_keys_kernel<<<grid_for(n, 256), 256, 0, s>>>(g.od.get(), n, maxod, bn, keys.get());
+    TC_LAUNCH_CHECK();
+    uint64_t *sorted = radix_sort_u64(keys.get(), tmp.get(), n, 0, kb, s);
+    g.perm.alloc(n, s);
+    perm_from_sorted_kernel<<<grid_for(n, 256), 256, 0, s>>>(sorted, n, (1ull << bn) - 1, g.perm.get());
+    TC_LAUNCH_CHECK();
+    g.identity_perm = false;
+  } else if (rule == TC_REORDER_PAPER) {
+    std::vector<uint32_t> h_od(n), h_perm;
+    if (n) TC_CUDA(cudaMemcpyAsync(h_od.data(), g.od.get(), sizeof(uint32_t) * n, cudaMemcpyDeviceToHost, s));
+    TC_CUDA(cudaStreamSynchronize(s));
+    aorder_host(h_od, p, h_perm, g.h_bucket_off, g.eq3);
+    if (n) {
+      g.perm.alloc(n, s);
+      TC_CUDA(cudaMemcpyAsync(g.perm.get(), h_perm.data(), sizeof(uint32_t) * n, cudaMemcpyHostToDevice, s));
+      g.identity_perm = false;
+    }
+    g.bucket_off.alloc(g.h_bucket_off.size(), s);
+    TC_CUDA(cudaMemcpyAsync(g.bucket_off.get(), g.h_bucket_off.data(), sizeof(uint32_t) * g.h_bucket_off.size(),
+                            cudaMemcpyHostToDevice, s));
+    TC_CUDA(cudaStreamSynchronize(s));  // host vectors must outlive the copies
+  }
+  g.reorder_rule = rule;
+  build_oriented_csr(g);
+  g.state = G_ORDERED;
+}
+
+}  // namespace tc

@@ -1,0 +1,250 @@
+"""GPU path vs the CPU oracle, element by element, through the C-ABI (libtc_b200.so).
+
+Bar: bit-exact for everything — T, per-vertex t(v), the
+simple graph, the orientation (out-degrees, A-direction subround/snapshot), the
+permutation, the A-order buckets and the oriented CSR.  Sizes span many radix
+tiles (4096 keys) with ragged tails; full-size configs are covered in
+test_gpu_configs.py.
+"""
+import itertools
+import zlib
+
+import numpy as np
+import pytest
+
+import graphgen
+import oracle
+import paper_conf_sigmod_hu0l21_b200 as tc
+from tests import graphs
+
+pytestmark = pytest.mark.gpu
+
+RULES = list(itertools.product(["id", "degree", "paper"], ["none", "degree", "paper"]))
+
+
+def _oracle_edges_u64(res):
+    return res["edges"]
+
+
+def check_against_oracle(src, dst, n, d, r, k=32, per_vertex=True, sched=None, order=0):
+    ref = oracle.run(src, dst, n, d, r, per_vertex=per_vertex, k=k, order=order)
+    g = tc.Graph(src, dst, n)
+    try:
+        edges, deg = g.export_graph()
+        assert np.array_equal(edges, ref["edges"]), "simple graph"
+        assert np.array_equal(deg, ref["deg"]), "degrees"
+        g.direct(d)
+        if d == "paper":
+            od, sub, dsnap = g.export_direct(internals=True)
+            assert np.array_equal(sub, ref["direct_info"]["sub"]), "A-direction subround"
+            assert np.array_equal(dsnap, ref["direct_info"]["dsnap"]), "A-direction snapshot"
+        else:
+            od = g.export_direct()
+        assert np.array_equal(od, ref["od"]), "out-degree"
+        g.reorder(r, k=k, order=order)
+        if sched:
+            g.set_schedule(sched)
+        offs, col, perm = g.export()
+        assert np.array_equal(perm, ref["perm"]), "permutation"
+        assert np.array_equal(offs, ref["offs"]), "CSR offsets"
+        assert np.array_equal(col, ref["col"]), "CSR columns"
+        if r == "paper":
+            assert np.array_equal(g.export_buckets(), ref["bucket_off"]), "A-order buckets"
+        if per_vertex:
+            T, t = g.count(per_vertex=True)
+            assert np.array_equal(t, ref["t"]), "per-vertex counts"
+        else:
+            T = g.count()
+        assert T == ref["T"], "triangle count"
+        st = g.stats()
+        assert st["m"] == ref["m"]
+        assert st["eq1"] == ref["eq1"]
+        return T, g.stats()
+    finally:
+        g.free()
+
+
+@pytest.mark.parametrize("name", sorted(graphs.CLOSED_FORMS))
+def test_closed_forms(name):
+    edges, n, T, t = graphs.CLOSED_FORMS[name]
+    rng = np.random.default_rng(zlib.crc32(name.encode()))
+    src, dst, N, perm = graphs.noisy_samples(edges, n, rng, pad=3)
+    t_expect = np.zeros(N, dtype=np.uint64)
+    t_expect[perm[:n]] = t
+    for d, r in RULES:
+        got, _ = check_against_oracle(src, dst, N, d, r, k=3)
+        assert got == T
+        g = tc.Graph(src, dst, N)
+        g.direct(d).reorder(r, k=3)
+        T2, tv = g.count(per_vertex=True)
+        assert T2 == T and np.array_equal(tv, t_expect)
+        g.free()
+
+
+@pytest.mark.parametrize("seed", range(40))
+def test_random_small(seed):
+    rng = np.random.default_rng(seed)
+    n = int(rng.integers(1, 3000))
+    M = int(rng.integers(0, 12 * n))
+    src, dst = graphs.random_graph(rng, n, M, "skew" if seed % 3 else "er")
+    d, r = RULES[seed % len(RULES)]
+    check_against_oracle(src, dst, n, d, r, k=int(rng.integers(1, 64)), order=seed % 2)
+
+
+@pytest.mark.parametrize("d,r", RULES)
+def test_config1_rmat_s16(d, r):
+    spec = graphgen.CONFIGS[1]
+    src, dst = graphgen.generate_cpu(spec)
+    check_against_oracle(src, dst, spec.n, d, r)
+
+
+@pytest.mark.parametrize("sched", ["bucketed", "range"])
+@pytest.mark.parametrize("cap", [32, 64, 1024])
+def test_schedules_and_caps(sched, cap):
+    """Every kernel path (warp slice, global-search fallback, CTA+TMA pieces) counts the same."""
+    spec = graphgen.rmat_spec(13, 16, 77)
+    src, dst = graphgen.generate_cpu(spec)
+    ref = oracle.run(src, dst, spec.n, "id", "none", per_vertex=True)
+    tc.tc_set_option("small_cap", cap)
+    try:
+        for d in ("id", "degree"):
+            g = tc.Graph(src, dst, spec.n).direct(d).reorder("none").set_schedule(sched)
+            T, t = g.count(per_vertex=True)
+            assert T == ref["T"] and np.array_equal(t, ref["t"])
+            g.free()
+    finally:
+        tc.tc_set_option("small_cap", 1024)
+
+
+def test_large_kernel_multi_piece():
+    """A star-heavy graph with ID directing: one source list > PIECE (16384) elements."""
+    rng = np.random.default_rng(9)
+    n = 40000
+    hub = 0
+    leaves = np.arange(1, n, dtype=np.uint32)
+    # hub -> every leaf, plus random leaf-leaf edges to make triangles through the hub
+    a = rng.integers(1, n, 60000).astype(np.uint32)
+    b = rng.integers(1, n, 60000).astype(np.uint32)
+    src = np.concatenate([np.full(n - 1, hub, np.uint32), a])
+    dst = np.concatenate([leaves, b])
+    ref = oracle.run(src, dst, n, "id", "none", per_vertex=True)
+    for sched in ("bucketed", "range"):
+        g = tc.Graph(src, dst, n).direct("id").reorder("none").set_schedule(sched)
+        T, t = g.count(per_vertex=True)
+        assert T == ref["T"] and np.array_equal(t, ref["t"])
+        g.free()
+
+
+def test_count_range_partition():
+    spec = graphgen.rmat_spec(14, 16, 5)
+    src, dst = graphgen.generate_cpu(spec)
+    for r in ("none", "paper"):
+        g = tc.Graph(src, dst, spec.n).direct("degree").reorder(r)
+        T = g.count()
+        for world in (1, 2, 3, 8):
+            b = g.partition(world)
+            assert b[0] == 0 and b[-1] == spec.n and np.all(np.diff(b.astype(np.int64)) >= 0)
+            parts = [g.count_range(int(b[i]), int(b[i + 1])) for i in range(world)]
+            assert sum(parts) == T
+        # per-vertex over a partition sums to the full per-vertex vector
+        T2, t = g.count(per_vertex=True)
+        b = g.partition(3)
+        acc = np.zeros(spec.n, np.uint64)
+        for i in range(3):
+            _, ti = g.count_range(int(b[i]), int(b[i + 1]), per_vertex=True)
+            acc += ti
+        assert np.array_equal(acc, t) and T2 == T
+        g.free()
+
+
+def test_device_and_host_inputs_agree():
+    import torch
+    spec = graphgen.rmat_spec(12, 16, 3)
+    src, dst = graphgen.generate_cpu(spec)
+    T_host = tc.count_triangles(src, dst, spec.n)
+    ds = torch.from_numpy(src.view(np.int32)).cuda()
+    dd = torch.from_numpy(dst.view(np.int32)).cuda()
+    g = tc.Graph(ds, dd, spec.n).direct("paper").reorder("paper")
+    assert g.count() == T_host
+    tv = torch.zeros(spec.n, dtype=torch.int64, device="cuda")
+    T_dev = tc.tc_count(g.handle, tv)
+    _, t_host = g.count(per_vertex=True)
+    assert T_dev == T_host and np.array_equal(tv.cpu().numpy().view(np.uint64), t_host)
+    g.free()
+
+
+def test_edge_cases():
+    z = np.zeros(0, np.uint32)
+    for n in (0, 1, 5):
+        g = tc.Graph(z, z, n).direct("paper").reorder("paper")
+        assert g.count() == 0
+        T, t = g.count(per_vertex=True)
+        assert T == 0 and (len(t) == 0 or t.sum() == 0)
+        g.free()
+    loops = np.array([1, 2, 2, 3], np.uint32)
+    assert tc.count_triangles(loops, loops, 4, "paper", "paper") == 0
+    one = np.array([0], np.uint32), np.array([1], np.uint32)
+    assert tc.count_triangles(*one, 2) == 0
+    tri = np.array([0, 1, 2], np.uint32), np.array([1, 2, 0], np.uint32)
+    assert tc.count_triangles(*tri, 3, "paper", "paper", per_vertex=True)[0] == 1
+
+
+def test_errors():
+    bad = np.array([0, 7], np.uint32)
+    with pytest.raises(tc.TCError) as e:
+        tc.Graph(bad, np.array([1, 1], np.uint32), 4)
+    assert e.value.status == tc.TC_ERR_INVALID
+    g = tc.Graph(np.array([0], np.uint32), np.array([1], np.uint32), 2)
+    with pytest.raises(tc.TCError) as e:
+        g.reorder("none")
+    assert e.value.status == tc.TC_ERR_STATE
+    with pytest.raises(tc.TCError) as e:
+        g.count()
+    assert e.value.status == tc.TC_ERR_STATE
+    g.direct("degree")
+    with pytest.raises(tc.TCError) as e:
+        g.reorder("paper", k=0)
+    assert e.value.status == tc.TC_ERR_INVALID
+    with pytest.raises(tc.TCError):
+        g.export_direct(internals=True)  # sub/dsnap only for PAPER
+    with pytest.raises(tc.TCError):
+        g.count_range(0, 5)
+    g.free()
+
+
+def test_redirect_resets_reorder():
+    spec = graphgen.rmat_spec(11, 16, 4)
+    src, dst = graphgen.generate_cpu(spec)
+    g = tc.Graph(src, dst, spec.n).direct("degree").reorder("paper")
+    T = g.count()
+    g.direct("paper")  # discards the reordering
+    offs, col, perm = g.export()
+    assert np.array_equal(perm, np.arange(spec.n))
+    assert g.count() == T
+    g.free()
+
+
+def test_aorder_params_bw_table_and_lpt():
+    spec = graphgen.rmat_spec(12, 16, 8)
+    src, dst = graphgen.generate_cpu(spec)
+    bw = np.linspace(1.0, 50.0, 64)
+    ref = oracle.run(src, dst, spec.n, "degree", "paper", k=16, lam=3.0, bw=bw, order=1)
+    g = tc.Graph(src, dst, spec.n).direct("degree").reorder("paper", k=16, lam=3.0, bw=bw, order=1)
+    offs, col, perm = g.export()
+    assert np.array_equal(perm, ref["perm"])
+    assert np.array_equal(g.export_buckets(), ref["bucket_off"])
+    assert g.stats()["eq3"] == oracle.objective_eq3(ref["bucket_off"], ref["perm"], ref["od"], lam=3.0, bw=bw)
+    assert g.count() == ref["T"]
+    g.free()
+
+
+def test_gpu_generator_matches_cpu():
+    import torch
+    for spec in (graphgen.rmat_spec(16, 4, 11), graphgen.er_spec(100003, 1 << 18, 12)):
+        s = torch.empty(spec.samples, dtype=torch.int32, device="cuda")
+        d = torch.empty(spec.samples, dtype=torch.int32, device="cuda")
+        graphgen.generate_cuda(spec, s.data_ptr(), d.data_ptr())
+        torch.cuda.synchronize()
+        cs, cd = graphgen.generate_cpu(spec)
+        assert np.array_equal(s.cpu().numpy().view(np.uint32), cs)
+        assert np.array_equal(d.cpu().numpy().view(np.uint32), cd)
