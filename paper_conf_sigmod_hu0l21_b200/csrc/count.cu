@@ -46,7 +46,7 @@ struct WarpScratch {  // per-warp owner-search tables for one 32-v chunk
 
 __device__ __forceinline__ uint32_t ldg_u32(const uint32_t *p) { return __ldg(p); }
 
-// Branchless search: does `w` occur in the ascending list s[0..L), L >= 1?
+// Branchless search: does `w` occur in the ascending list s[0..L), L >= 1? (any memory)
 __device__ __forceinline__ bool bsearch_list(const uint32_t *s, uint32_t L, uint32_t w) {
   const uint32_t *p = s;
   uint32_t len = L;
@@ -58,12 +58,66 @@ __device__ __forceinline__ bool bsearch_list(const uint32_t *s, uint32_t L, uint
   return *p == w;
 }
 
-// Count the wedges u->v->w of one chunk of up to 32 v's (lane-held `v`, `valid`) whose
-// w lies in list[0..L) (w restricted to [lo, hi]).  Returns this lane's matches.
+// Fixed-depth search over a list padded with +inf (0xffffffff, never a vertex id) to 2^S
+// entries: S unrolled steps of one shared load + compare + select each ("binary lifting").
+// Precondition: s[0] <= w (the caller's range filter).
+template <int S>
+__device__ __forceinline__ bool bsearch_pow2(const uint32_t *s, uint32_t w) {
+  uint32_t p = 0;
+#pragma unroll
+  for (int k = S - 1; k >= 0; --k) {
+    uint32_t q = p + (1u << k);
+    p = (s[q] <= w) ? q : p;
+  }
+  return s[p] == w;
+}
+
+__device__ __forceinline__ int ceil_log2(uint32_t L) { return L <= 1 ? 0 : 32 - __clz(L - 1); }
+
+// Wedge loop of one chunk.  Owner tables hold only the non-empty N+(v) of the chunk
+// (K entries: start offset, inclusive wedge prefix); each lane walks its owner forward
+// incrementally (its wedge index grows by 32 per step), so locating w's list costs ~1
+// shared load per wedge instead of a 5-step search.
+template <bool PV, int S>
+__device__ __forceinline__ uint32_t wedge_loop(const uint32_t *__restrict__ col, const uint32_t *list, uint32_t L,
+                                               uint32_t lo, uint32_t hi, uint32_t total, const WarpScratch &ws,
+                                               unsigned long long *tv) {
+  uint32_t cnt = 0;
+  uint32_t o = 0, o_beg = 0, o_end = ws.pre[0];
+  uint64_t o_vb = ws.vb[0];
+  for (uint32_t j = lane_id(); j < total; j += 32) {
+    if (o_end <= j) {
+      do {
+        ++o;
+        o_beg = o_end;
+        o_end = ws.pre[o];
+      } while (o_end <= j);
+      o_vb = ws.vb[o];
+    }
+    const uint32_t w = ldg_u32(col + o_vb + (j - o_beg));
+    if (w >= lo && w <= hi) {
+      bool hit;
+      if (S > 0) hit = bsearch_pow2<S>(list, w);
+      else hit = bsearch_list(list, L, w);
+      if (hit) {
+        ++cnt;
+        if (PV) {
+          atomicAdd(&tv[w], 1ull);
+          atomicAdd(&tv[ws.v[o]], 1ull);
+        }
+      }
+    }
+  }
+  return cnt;
+}
+
+// Count the wedges u->v->w of one chunk of up to 32 v's (lane-held `v`, `valid`) whose w
+// lies in list[0..L) (w restricted to [lo, hi]).  `padded`: list is padded with +inf to
+// 2^ceil(log2 L) entries (shared-memory copies).  Returns this lane's matches.
 template <bool PV>
 __device__ __forceinline__ uint32_t warp_chunk(const uint64_t *__restrict__ offs, const uint32_t *__restrict__ col,
-                                               uint32_t v, bool valid, const uint32_t *list, uint32_t L, uint32_t lo,
-                                               uint32_t hi, WarpScratch &ws, unsigned long long *tv) {
+                                               uint32_t v, bool valid, const uint32_t *list, uint32_t L, bool padded,
+                                               uint32_t lo, uint32_t hi, WarpScratch &ws, unsigned long long *tv) {
   const unsigned lane = lane_id();
   uint64_t vb = 0;
   uint32_t dv = 0;
@@ -71,62 +125,67 @@ __device__ __forceinline__ uint32_t warp_chunk(const uint64_t *__restrict__ offs
     vb = offs[v];
     dv = (uint32_t)(offs[v + 1] - vb);
   }
-  uint32_t inc = warp_inclusive_scan(dv);
-  uint32_t total = __shfl_sync(0xffffffffu, inc, 31);
-  ws.vb[lane] = vb;
-  ws.pre[lane] = inc;
-  if (PV) ws.v[lane] = v;
+  const uint32_t inc = warp_inclusive_scan(dv);
+  const uint32_t total = __shfl_sync(0xffffffffu, inc, 31);
+  const unsigned nz = __ballot_sync(0xffffffffu, dv != 0);
+  if (dv) {
+    const unsigned pos = __popc(nz & ((1u << lane) - 1u));
+    ws.vb[pos] = vb;
+    ws.pre[pos] = inc;
+    if (PV) ws.v[pos] = v;
+  }
   __syncwarp();
   uint32_t cnt = 0;
-  for (uint32_t j = lane; j < total; j += 32) {
-    uint32_t o = 0;
-#pragma unroll
-    for (uint32_t step = 16; step; step >>= 1) o = (ws.pre[o + step - 1] <= j) ? o + step : o;
-    uint32_t excl = o ? ws.pre[o - 1] : 0u;
-    uint32_t w = ldg_u32(col + ws.vb[o] + (j - excl));
-    if (w >= lo && w <= hi && bsearch_list(list, L, w)) {
-      ++cnt;
-      if (PV) {
-        atomicAdd(&tv[w], 1ull);
-        atomicAdd(&tv[ws.v[o]], 1ull);
-      }
+  if (total) {
+    const int S = padded ? ceil_log2(L) : 0;
+    switch (S) {
+#define TC_CASE(k) \
+  case k:          \
+    cnt = wedge_loop<PV, k>(col, list, L, lo, hi, total, ws, tv); \
+    break;
+      TC_CASE(1) TC_CASE(2) TC_CASE(3) TC_CASE(4) TC_CASE(5) TC_CASE(6) TC_CASE(7)
+      TC_CASE(8) TC_CASE(9) TC_CASE(10) TC_CASE(11) TC_CASE(12) TC_CASE(13) TC_CASE(14)
+#undef TC_CASE
+      default:
+        cnt = wedge_loop<PV, 0>(col, list, L, lo, hi, total, ws, tv);
     }
   }
   __syncwarp();
   return cnt;
 }
 
-// Process source vertex u with one warp; list = shared slice (SMEM) or global N+(u).
+// One work item: source u, v's N+(u)[c0 .. c0+32) on one warp; N+(u) is searched in the
+// warp's shared slice (staged here, padded with +inf to a power of two) when it fits,
+// else in global memory.
 template <bool PV>
-__device__ __forceinline__ uint64_t warp_vertex(const uint64_t *__restrict__ offs, const uint32_t *__restrict__ col,
-                                                uint32_t u, uint32_t *slice, uint32_t cap, WarpScratch &ws,
-                                                unsigned long long *tv) {
+__device__ __forceinline__ uint64_t warp_item(const uint64_t *__restrict__ offs, const uint32_t *__restrict__ col,
+                                              uint32_t u, uint32_t c0, uint32_t *slice, uint32_t cap,
+                                              WarpScratch &ws, unsigned long long *tv) {
   const unsigned lane = lane_id();
   const uint64_t a = offs[u];
   const uint32_t L = (uint32_t)(offs[u + 1] - a);
-  if (L < 2) return 0;
+  if (L < 2 || c0 >= L) return 0;
   const uint32_t *list;
+  bool padded = false;
   if (L <= cap) {
-    for (uint32_t j = lane; j < L; j += 32) slice[j] = ldg_u32(col + a + j);
+    const uint32_t P = 1u << ceil_log2(L);
+    for (uint32_t j = lane; j < P; j += 32) slice[j] = j < L ? ldg_u32(col + a + j) : 0xffffffffu;
     __syncwarp();
     list = slice;
+    padded = true;
   } else {
     list = col + a;
   }
   const uint32_t lo = list[0], hi = list[L - 1];
-  uint32_t cnt = 0;
-  for (uint32_t c0 = 0; c0 < L; c0 += 32) {
-    bool valid = c0 + lane < L;
-    uint32_t v = valid ? list[c0 + lane] : 0u;
-    cnt += warp_chunk<PV>(offs, col, v, valid, list, L, lo, hi, ws, tv);
-  }
-  __syncwarp();
-  uint64_t c = cnt;
+  const bool valid = c0 + lane < L;
+  const uint32_t v = valid ? list[c0 + lane] : 0u;
+  uint32_t cnt = warp_chunk<PV>(offs, col, v, valid, list, L, padded, lo, hi, ws, tv);
+  __syncwarp();  // slice reads done before the next item restages it
   if (PV) {
-    uint64_t tot = warp_sum(c);
+    uint64_t tot = warp_sum((uint64_t)cnt);
     if (lane == 0 && tot) atomicAdd(&tv[u], (unsigned long long)tot);
   }
-  return c;
+  return cnt;
 }
 
 __device__ __forceinline__ void block_add_u64(uint64_t v, unsigned long long *T) {
@@ -143,63 +202,108 @@ __device__ __forceinline__ void block_add_u64(uint64_t v, unsigned long long *T)
 }
 
 // --------------------------------------------------------------- schedule (a8)
+// Work items (u, c0): N+(u) is cut into chunks of SV = 32 v's (warp items, d~(u) < cap) or
+// LV = 512 v's (CTA items, d~(u) >= cap), so one heavy source never serialises on one
+// warp.  Items are grouped in floor(log2 d~(u)) bins, heaviest bin first (cf. the
+// logarithmic radix binning of P:63); within a bin the order is arbitrary (counts are
+// order-independent integers).
+constexpr uint32_t SV = 32;
+constexpr uint32_t LV = LG_THREADS;
+
 __device__ __forceinline__ int deg_bin(uint32_t d) { return 31 - __clz(d); }  // floor(log2 d), d >= 1
 
-__global__ void bin_hist_kernel(const uint64_t *__restrict__ offs, uint32_t ub, uint32_t ue, unsigned *hist) {
-  __shared__ unsigned s_h[32];
+__device__ __forceinline__ uint32_t items_of(uint32_t d, uint32_t cap) {
+  if (d < 2) return 0;
+  return d < cap ? (d + SV - 1) / SV : (d + LV - 1) / LV;
+}
+
+__global__ void items_hist_kernel(const uint64_t *__restrict__ offs, uint32_t ub, uint32_t ue, uint32_t cap,
+                                  unsigned long long *hist) {
+  __shared__ unsigned long long s_h[32];
   if (threadIdx.x < 32) s_h[threadIdx.x] = 0;
   __syncthreads();
   for (uint64_t u = (uint64_t)ub + blockIdx.x * blockDim.x + threadIdx.x; u < ue; u += (uint64_t)gridDim.x * blockDim.x) {
     uint32_t d = (uint32_t)(offs[u + 1] - offs[u]);
-    if (d >= 2) atomicAdd(&s_h[deg_bin(d)], 1u);
+    uint32_t it = items_of(d, cap);
+    if (it) atomicAdd(&s_h[deg_bin(d)], (unsigned long long)it);
   }
   __syncthreads();
   if (threadIdx.x < 32 && s_h[threadIdx.x]) atomicAdd(&hist[threadIdx.x], s_h[threadIdx.x]);
 }
 
-// cursor[bin] = start of bin in the worklist, bins in DESCENDING order (heaviest first)
-__global__ void bin_scan_kernel(const unsigned *hist, unsigned *cursor) {
+// cursor[bin] = start of bin in the item list, bins in DESCENDING order (heaviest first)
+__global__ void bin_scan_kernel(const unsigned long long *hist, unsigned long long *cursor) {
   unsigned lane = threadIdx.x;  // 32 threads; lane = 31 - bin
-  unsigned c = hist[31 - lane];
-  unsigned inc = warp_inclusive_scan(c);
+  unsigned long long c = hist[31 - lane];
+  unsigned long long inc = warp_inclusive_scan(c);
   cursor[31 - lane] = inc - c;
 }
 
-__global__ void bin_scatter_kernel(const uint64_t *__restrict__ offs, uint32_t ub, uint32_t ue, unsigned *cursor,
-                                   uint32_t *__restrict__ work) {
-  uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-  for (uint64_t base = (uint64_t)ub + blockIdx.x * blockDim.x + (threadIdx.x & ~31u); base < ue; base += stride) {
-    uint64_t u = base + lane_id();
-    uint32_t d = u < ue ? (uint32_t)(offs[u + 1] - offs[u]) : 0u;
-    int bin = d >= 2 ? deg_bin(d) : -1;
-    unsigned peers = __match_any_sync(0xffffffffu, bin);
-    unsigned leader = __ffs(peers) - 1;
-    unsigned pos = 0;
-    if (bin >= 0 && lane_id() == leader) pos = atomicAdd(&cursor[bin], (unsigned)__popc(peers));
-    pos = __shfl_sync(0xffffffffu, pos, leader);
-    if (bin >= 0) work[pos + __popc(peers & ((1u << lane_id()) - 1u))] = (uint32_t)u;
+constexpr int SC_PER_THREAD = 8;
+__global__ __launch_bounds__(256) void items_scatter_kernel(const uint64_t *__restrict__ offs, uint32_t ub,
+                                                            uint32_t ue, uint32_t cap, unsigned long long *cursor,
+                                                            uint64_t *__restrict__ items) {
+  __shared__ unsigned s_cnt[32];
+  __shared__ unsigned long long s_base[32];
+  const uint64_t span = 256ull * SC_PER_THREAD;
+  for (uint64_t c0 = (uint64_t)ub + blockIdx.x * span; c0 < ue; c0 += (uint64_t)gridDim.x * span) {
+    if (threadIdx.x < 32) s_cnt[threadIdx.x] = 0;
+    __syncthreads();
+    uint32_t off[SC_PER_THREAD], d[SC_PER_THREAD];
+#pragma unroll
+    for (int i = 0; i < SC_PER_THREAD; ++i) {
+      uint64_t u = c0 + (uint64_t)i * 256 + threadIdx.x;
+      d[i] = u < ue ? (uint32_t)(offs[u + 1] - offs[u]) : 0u;
+      uint32_t it = items_of(d[i], cap);
+      off[i] = it ? atomicAdd(&s_cnt[deg_bin(d[i])], it) : 0u;
+    }
+    __syncthreads();
+    if (threadIdx.x < 32) s_base[threadIdx.x] = s_cnt[threadIdx.x] ? atomicAdd(&cursor[threadIdx.x], (unsigned long long)s_cnt[threadIdx.x]) : 0ull;
+    __syncthreads();
+#pragma unroll
+    for (int i = 0; i < SC_PER_THREAD; ++i) {
+      uint32_t it = items_of(d[i], cap);
+      if (!it) continue;
+      uint64_t u = c0 + (uint64_t)i * 256 + threadIdx.x;
+      uint64_t p = s_base[deg_bin(d[i])] + off[i];
+      uint32_t step = d[i] < cap ? SV : LV;
+      for (uint32_t c = 0; c < it; ++c) items[p + c] = (u << 32) | (uint64_t)(c * step);
+    }
+    __syncthreads();
   }
 }
 
 // --------------------------------------------------------------- count kernels (a9)
+// Warp items; items [0, nheavy) are fetched one at a time, the rest CHUNK at a time.
 template <bool PV>
 __global__ __launch_bounds__(CT_THREADS) void count_small_kernel(const uint64_t *__restrict__ offs,
                                                                  const uint32_t *__restrict__ col,
-                                                                 const uint32_t *__restrict__ work, uint32_t nwork,
-                                                                 unsigned *work_ctr, uint32_t cap,
+                                                                 const uint64_t *__restrict__ items, uint64_t nitems,
+                                                                 uint64_t nheavy, unsigned long long *ctr, uint32_t cap,
                                                                  unsigned long long *T, unsigned long long *tv) {
   extern __shared__ uint32_t s_dyn[];
   __shared__ WarpScratch s_ws[CT_WARPS];
   uint32_t *slice = s_dyn + warp_id() * cap;
   WarpScratch &ws = s_ws[warp_id()];
   uint64_t acc = 0;
-  while (true) {
-    unsigned base = 0;
-    if (lane_id() == 0) base = atomicAdd(work_ctr, CHUNK);
-    base = __shfl_sync(0xffffffffu, base, 0);
-    if (base >= nwork) break;
-    unsigned end = min(base + CHUNK, nwork);
-    for (unsigned i = base; i < end; ++i) acc += warp_vertex<PV>(offs, col, work[i], slice, cap, ws, tv);
+  while (true) {  // heavy items, one per fetch
+    unsigned long long i = 0;
+    if (lane_id() == 0) i = atomicAdd(&ctr[0], 1ull);
+    i = __shfl_sync(0xffffffffu, i, 0);
+    if (i >= nheavy) break;
+    uint64_t it = items[i];
+    acc += warp_item<PV>(offs, col, (uint32_t)(it >> 32), (uint32_t)it, slice, cap, ws, tv);
+  }
+  while (true) {  // light items, CHUNK per fetch
+    unsigned long long b = 0;
+    if (lane_id() == 0) b = nheavy + atomicAdd(&ctr[1], (unsigned long long)CHUNK);
+    b = __shfl_sync(0xffffffffu, b, 0);
+    if (b >= nitems) break;
+    uint64_t e = min((uint64_t)b + CHUNK, nitems);
+    for (uint64_t i = b; i < e; ++i) {
+      uint64_t it = items[i];
+      acc += warp_item<PV>(offs, col, (uint32_t)(it >> 32), (uint32_t)it, slice, cap, ws, tv);
+    }
   }
   block_add_u64(acc, T);
 }
@@ -233,31 +337,34 @@ __device__ __forceinline__ void mbar_wait(uint64_t *bar, unsigned phase) {
       : "memory");
 }
 
-// CTA per heavy source vertex; N+(u) staged piece by piece with a TMA bulk copy.
+// CTA items (u, c0) of heavy sources: v's N+(u)[c0 .. c0+LV) over 16 warps; N+(u) staged
+// piece by piece with a TMA bulk copy (cp.async.bulk + mbarrier complete_tx).
 template <bool PV>
 __global__ __launch_bounds__(LG_THREADS) void count_large_kernel(const uint64_t *__restrict__ offs,
                                                                  const uint32_t *__restrict__ col,
-                                                                 const uint32_t *__restrict__ work, uint32_t nwork,
-                                                                 unsigned *work_ctr, unsigned long long *T,
+                                                                 const uint64_t *__restrict__ items, uint64_t nitems,
+                                                                 unsigned long long *ctr, unsigned long long *T,
                                                                  unsigned long long *tv) {
   extern __shared__ __align__(128) uint32_t s_piece[];  // PIECE + 8 words (alignment slack)
   __shared__ WarpScratch s_ws[LG_WARPS];
   __shared__ __align__(8) uint64_t s_bar;
-  __shared__ unsigned s_item;
+  __shared__ unsigned long long s_item;
   WarpScratch &ws = s_ws[warp_id()];
   if (threadIdx.x == 0) mbar_init(&s_bar, 1);
   __syncthreads();
   unsigned phase = 0;
   uint64_t acc = 0;
   while (true) {
-    if (threadIdx.x == 0) s_item = atomicAdd(work_ctr, 1u);
+    if (threadIdx.x == 0) s_item = atomicAdd(ctr, 1ull);
     __syncthreads();
-    unsigned item = s_item;
+    unsigned long long item = s_item;
     __syncthreads();
-    if (item >= nwork) break;
-    const uint32_t u = work[item];
+    if (item >= nitems) break;
+    const uint64_t it = items[item];
+    const uint32_t u = (uint32_t)(it >> 32), cbeg = (uint32_t)it;
     const uint64_t a = offs[u];
     const uint32_t L = (uint32_t)(offs[u + 1] - a);
+    const uint32_t cend = min(L, cbeg + LV);
     uint64_t ucnt = 0;
     for (uint32_t p0 = 0; p0 < L; p0 += PIECE) {
       const uint32_t plen = min(PIECE, L - p0);
@@ -275,12 +382,17 @@ __global__ __launch_bounds__(LG_THREADS) void count_large_kernel(const uint64_t 
       mbar_wait(&s_bar, phase);
       phase ^= 1u;
       const uint32_t *list = s_piece + shift;
+      {  // pad the piece with +inf up to a power of two for the fixed-depth search
+        const uint32_t P = 1u << ceil_log2(plen);
+        for (uint32_t j = plen + threadIdx.x; j < P; j += LG_THREADS) s_piece[shift + j] = 0xffffffffu;
+        __syncthreads();
+      }
       const uint32_t lo = list[0], hi = list[plen - 1];
       uint32_t cnt = 0;
-      for (uint32_t c0 = warp_id() * 32; c0 < L; c0 += LG_THREADS) {
-        bool valid = c0 + lane_id() < L;
+      for (uint32_t c0 = cbeg + warp_id() * 32; c0 < cend; c0 += LG_THREADS) {
+        bool valid = c0 + lane_id() < cend;
         uint32_t v = valid ? ldg_u32(col + a + c0 + lane_id()) : 0u;
-        cnt += warp_chunk<PV>(offs, col, v, valid, list, plen, lo, hi, ws, tv);
+        cnt += warp_chunk<PV>(offs, col, v, valid, list, plen, true, lo, hi, ws, tv);
       }
       ucnt += cnt;
       __syncthreads();  // piece fully consumed before the next bulk copy overwrites it
@@ -312,8 +424,17 @@ __global__ __launch_bounds__(CT_THREADS) void count_range_kernel(const uint64_t 
     uint64_t s1 = boff ? boff[bi + 1] : (uint64_t)(bi + 1) * kfixed;
     if (s0 < ub) s0 = ub;
     if (s1 > ue) s1 = ue;
-    for (uint64_t u = s0 + warp_id(); u < s1; u += CT_WARPS)
-      acc += warp_vertex<PV>(offs, col, (uint32_t)u, slice, cap, ws, tv);
+    // the bucket's (u, 32-v chunk) items, dealt round-robin to the CTA's warps
+    uint32_t t = 0;
+    for (uint64_t u = s0; u < s1; ++u) {
+      uint32_t L = (uint32_t)(offs[u + 1] - offs[u]);
+      if (L < 2) continue;
+      uint32_t nit = (L + SV - 1) / SV;
+      uint32_t first = (warp_id() + CT_WARPS - (t % CT_WARPS)) % CT_WARPS;
+      for (uint32_t c = first; c < nit; c += CT_WARPS)
+        acc += warp_item<PV>(offs, col, (uint32_t)u, c * SV, slice, cap, ws, tv);
+      t += nit;
+    }
   }
   block_add_u64(acc, T);
 }
@@ -443,30 +564,35 @@ uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *
         ++nlaunch;
       }
     } else {
-      // degree-binned worklist (heaviest bin first)
-      DevBuf<unsigned> hist;  // [0..31] hist, [32..63] cursor, [64] small ctr, [65] large ctr
-      hist.alloc(66, s);
+      // degree-binned item list (heaviest bin first)
+      DevBuf<unsigned long long> hist;  // [0..31] items/bin, [32..63] cursor, [64..66] fetch counters
+      hist.alloc(67, s);
       TC_CUDA(cudaMemsetAsync(hist.get(), 0, hist.bytes(), s));
-      bin_hist_kernel<<<grid_for(ue - ub, 256, 4), 256, 0, s>>>(g.offs.get(), ub, ue, hist.get());
+      items_hist_kernel<<<grid_for(ue - ub, 256, 4), 256, 0, s>>>(g.offs.get(), ub, ue, cap, hist.get());
       TC_LAUNCH_CHECK();
       bin_scan_kernel<<<1, 32, 0, s>>>(hist.get(), hist.get() + 32);
       TC_LAUNCH_CHECK();
-      std::vector<unsigned> hh(32);
-      TC_CUDA(cudaMemcpyAsync(hh.data(), hist.get(), 32 * sizeof(unsigned), cudaMemcpyDeviceToHost, s));
+      std::vector<unsigned long long> hh(32);
+      TC_CUDA(cudaMemcpyAsync(hh.data(), hist.get(), 32 * sizeof(unsigned long long), cudaMemcpyDeviceToHost, s));
       TC_CUDA(cudaStreamSynchronize(s));
-      uint64_t nwork = 0, nlarge = 0;
-      int capbin = 31 - __builtin_clz(cap);  // d < cap  <=>  bin < capbin
+      uint64_t nitems = 0, nlarge = 0, nheavy = 0;
+      const int capbin = 31 - __builtin_clz(cap);  // d < cap  <=>  bin < capbin
       for (int b = 0; b < 32; ++b) {
-        nwork += hh[b];
+        nitems += hh[b];
         if (b >= capbin) nlarge += hh[b];
+        else if (b >= 5) nheavy += hh[b];  // d~ >= 32: fetched one item at a time
       }
-      nlaunch += 3;
-      if (nwork) {
-        DevBuf<uint32_t> work;
-        work.alloc(nwork, s);
-        bin_scatter_kernel<<<grid_for(ue - ub, 256), 256, 0, s>>>(g.offs.get(), ub, ue, hist.get() + 32, work.get());
-        TC_LAUNCH_CHECK();
-        ++nlaunch;
+      nlaunch += 2;
+      if (nitems) {
+        DevBuf<uint64_t> items;
+        items.alloc(nitems, s);
+        {
+          uint64_t span = 256ull * SC_PER_THREAD;
+          unsigned grid = (unsigned)std::min<uint64_t>((ue - ub + span - 1) / span, (uint64_t)num_sms() * 8);
+          items_scatter_kernel<<<grid, 256, 0, s>>>(g.offs.get(), ub, ue, cap, hist.get() + 32, items.get());
+          TC_LAUNCH_CHECK();
+          ++nlaunch;
+        }
         if (kernel_ms) TC_CUDA(cudaEventRecord(e0, s));
         if (nlarge) {
           size_t smem = (PIECE + 8) * sizeof(uint32_t);
@@ -475,29 +601,28 @@ uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *
           unsigned grid = (unsigned)std::min<uint64_t>(nlarge, (uint64_t)num_sms() * occ);
           ProfScope prof("count_large", s, 0.0);
           if (tv)
-            count_large_kernel<true><<<grid, LG_THREADS, smem, s>>>(g.offs.get(), g.col.get(), work.get(),
-                                                                     (uint32_t)nlarge, hist.get() + 65, dT.get(), tv);
+            count_large_kernel<true><<<grid, LG_THREADS, smem, s>>>(g.offs.get(), g.col.get(), items.get(), nlarge,
+                                                                     hist.get() + 64, dT.get(), tv);
           else
-            count_large_kernel<false><<<grid, LG_THREADS, smem, s>>>(g.offs.get(), g.col.get(), work.get(),
-                                                                      (uint32_t)nlarge, hist.get() + 65, dT.get(),
-                                                                      nullptr);
+            count_large_kernel<false><<<grid, LG_THREADS, smem, s>>>(g.offs.get(), g.col.get(), items.get(), nlarge,
+                                                                      hist.get() + 64, dT.get(), nullptr);
           TC_LAUNCH_CHECK();
           ++nlaunch;
         }
-        uint64_t nsmall = nwork - nlarge;
+        uint64_t nsmall = nitems - nlarge;
         if (nsmall) {
           size_t smem = (size_t)CT_WARPS * cap * sizeof(uint32_t);
           int occ = occupancy(tv ? (const void *)count_small_kernel<true> : (const void *)count_small_kernel<false>,
                               CT_THREADS, smem);
-          uint64_t want = (nsmall + CT_WARPS * CHUNK - 1) / (CT_WARPS * CHUNK);
+          uint64_t want = (nsmall + CT_WARPS - 1) / CT_WARPS;
           unsigned grid = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(want, (uint64_t)num_sms() * occ));
           ProfScope prof("count_small", s, 0.0);
           if (tv)
-            count_small_kernel<true><<<grid, CT_THREADS, smem, s>>>(g.offs.get(), g.col.get(), work.get() + nlarge,
-                                                                     (uint32_t)nsmall, hist.get() + 64, cap, dT.get(), tv);
+            count_small_kernel<true><<<grid, CT_THREADS, smem, s>>>(g.offs.get(), g.col.get(), items.get() + nlarge,
+                                                                     nsmall, nheavy, hist.get() + 65, cap, dT.get(), tv);
           else
-            count_small_kernel<false><<<grid, CT_THREADS, smem, s>>>(g.offs.get(), g.col.get(), work.get() + nlarge,
-                                                                      (uint32_t)nsmall, hist.get() + 64, cap, dT.get(),
+            count_small_kernel<false><<<grid, CT_THREADS, smem, s>>>(g.offs.get(), g.col.get(), items.get() + nlarge,
+                                                                      nsmall, nheavy, hist.get() + 65, cap, dT.get(),
                                                                       nullptr);
           TC_LAUNCH_CHECK();
           ++nlaunch;

@@ -124,13 +124,35 @@ __global__ void rs_hist_scan_kernel(unsigned long long *ghist, int passes) {
   }
 }
 
-__global__ __launch_bounds__(T_THREADS) void rs_pass_kernel(const uint64_t *__restrict__ in,
-                                                            uint64_t *__restrict__ out, uint64_t n,
-                                                            int shift,
-                                                            const unsigned long long *__restrict__ goff,
-                                                            uint64_t *status, uint32_t *tile_ctr) {
+// Stable rank of one warp-striped item across the warp: lanes with equal digit found with
+// 8 ballots (cheaper than match.any on sm_100a's MIO pipe), the group leader bumps the
+// warp's smem counter once, the old value is broadcast back.  Items are processed in
+// order by the same warp, so equal digits keep input order (LSD stability).
+template <bool FULL>
+__device__ __forceinline__ uint32_t rank_item(uint32_t d, bool valid, uint32_t *whist, unsigned lt_mask) {
+  unsigned peers = FULL ? 0xffffffffu : __ballot_sync(0xffffffffu, valid);
+  if (!FULL && !valid) peers = ~peers;
+#pragma unroll
+  for (int b = 0; b < 8; ++b) {
+    unsigned bit = (d >> b) & 1u;
+    unsigned bb = __ballot_sync(0xffffffffu, bit);
+    peers &= bit ? bb : ~bb;
+  }
+  unsigned lead = __ffs(peers) - 1;
+  uint32_t old = 0;
+  if (lane_id() == lead && (FULL || valid)) old = atomicAdd(&whist[d], (uint32_t)__popc(peers));
+  old = __shfl_sync(0xffffffffu, old, lead);
+  return old + __popc(peers & lt_mask);
+}
+
+__global__ __launch_bounds__(T_THREADS, 3) void rs_pass_kernel(const uint64_t *__restrict__ in,
+                                                               uint64_t *__restrict__ out, uint64_t n,
+                                                               int shift,
+                                                               const unsigned long long *__restrict__ goff,
+                                                               uint64_t *status, uint32_t *tile_ctr) {
   __shared__ uint64_t s_keys[T_TILE];
   __shared__ uint32_t s_whist[T_WARPS][256];
+  __shared__ uint32_t s_cnt[256];
   __shared__ uint32_t s_lstart[256];
   __shared__ uint64_t s_gbase[256];
   __shared__ uint32_t s_warp32[8];
@@ -140,33 +162,44 @@ __global__ __launch_bounds__(T_THREADS) void rs_pass_kernel(const uint64_t *__re
   if (t == 0) s_tile = atomicAdd(tile_ctr, 1u);
 #pragma unroll
   for (int i = 0; i < T_WARPS; ++i) s_whist[i][t] = 0;
+  s_cnt[t] = 0;
   __syncthreads();
   const uint64_t tile = s_tile;
   const uint64_t base = tile * T_TILE;
+  const bool full = base + T_TILE <= n;
 
   uint64_t k[T_ITEMS];
-  uint32_t d[T_ITEMS];
   uint32_t r[T_ITEMS];
+  const uint64_t wbase = base + w * (32 * T_ITEMS) + l;  // warp-striped: stable order
+  if (full) {
 #pragma unroll
-  for (int i = 0; i < T_ITEMS; ++i) {
-    uint64_t idx = base + w * (32 * T_ITEMS) + i * 32 + l;  // warp-striped: stable order
-    bool valid = idx < n;
-    k[i] = valid ? in[idx] : ~0ull;
-    d[i] = valid ? (uint32_t)((k[i] >> shift) & 255u) : 256u;
+    for (int i = 0; i < T_ITEMS; ++i) k[i] = __ldcs(in + wbase + i * 32);
+  } else {
+#pragma unroll
+    for (int i = 0; i < T_ITEMS; ++i) k[i] = (wbase + i * 32 < n) ? in[wbase + i * 32] : ~0ull;
   }
-  const unsigned lt_mask = (1u << l) - 1u;
+  // early tile histogram -> publish the aggregate before the (long) ranking so that
+  // successors' look-back rarely waits (one-sweep "early counts")
 #pragma unroll
-  for (int i = 0; i < T_ITEMS; ++i) {
-    unsigned peers = __match_any_sync(0xffffffffu, d[i]);
-    unsigned lead = __ffs(peers) - 1;
-    uint32_t cur = d[i] < 256u ? s_whist[w][d[i]] : 0u;
-    r[i] = cur + __popc(peers & lt_mask);
-    __syncwarp();
-    if (l == lead && d[i] < 256u) s_whist[w][d[i]] = cur + __popc(peers);
-    __syncwarp();
+  for (int i = 0; i < T_ITEMS; ++i)
+    if (full || wbase + i * 32 < n) atomicAdd(&s_cnt[(uint32_t)(k[i] >> shift) & 255u], 1u);
+  __syncthreads();
+  const uint32_t tcount = s_cnt[t];
+  uint64_t *st = status + t;  // status laid out [tile][256]
+  st_relaxed_u64(st + tile * 256, (tile == 0 ? LB_INC : LB_AGG) | tcount);
+
+  const unsigned lt_mask = (1u << l) - 1u;
+  uint32_t *whist = s_whist[w];
+  if (full) {
+#pragma unroll
+    for (int i = 0; i < T_ITEMS; ++i) r[i] = rank_item<true>((uint32_t)(k[i] >> shift) & 255u, true, whist, lt_mask);
+  } else {
+#pragma unroll
+    for (int i = 0; i < T_ITEMS; ++i)
+      r[i] = rank_item<false>((uint32_t)(k[i] >> shift) & 255u, wbase + i * 32 < n, whist, lt_mask);
   }
   __syncthreads();
-  // digit t: exclusive prefix over warps, tile count
+  // digit t: exclusive prefix over warps
   uint32_t run = 0;
 #pragma unroll
   for (int ww = 0; ww < T_WARPS; ++ww) {
@@ -174,33 +207,39 @@ __global__ __launch_bounds__(T_THREADS) void rs_pass_kernel(const uint64_t *__re
     s_whist[ww][t] = run;
     run += c;
   }
-  uint32_t lstart = block256_exclusive_scan<uint32_t>(run, s_warp32, &s_total32);
+  uint32_t lstart = block256_exclusive_scan<uint32_t>(tcount, s_warp32, &s_total32);
   s_lstart[t] = lstart;
-  // look-back for digit t (status laid out [tile][256])
-  {
-    uint64_t *st = status + t;
-    uint64_t e = 0;
-    if (tile == 0) {
-      st_relaxed_u64(st, LB_INC | run);
-    } else {
-      st_relaxed_u64(st + tile * 256, LB_AGG | run);
-      int64_t j = (int64_t)tile - 1;
-      while (true) {
-        uint64_t sv = ld_relaxed_u64(st + (uint64_t)j * 256);
-        uint64_t f = sv & ~LB_VAL;
+  // look-back for digit t, four predecessors per round trip
+  uint64_t e = 0;
+  if (tile > 0) {
+    int64_t j = (int64_t)tile - 1;
+    while (true) {
+      uint64_t v[4];
+#pragma unroll
+      for (int q = 0; q < 4; ++q) v[q] = (j - q >= 0) ? ld_relaxed_u64(st + (uint64_t)(j - q) * 256) : 0ull;
+      int q = 0;
+      bool done = false;
+#pragma unroll
+      for (int qq = 0; qq < 4; ++qq) {
+        if (done || q != qq || j - qq < 0) continue;
+        uint64_t f = v[qq] & ~LB_VAL;
         if (f == 0) continue;
-        e += sv & LB_VAL;
-        if (f == LB_INC) break;
-        --j;
+        e += v[qq] & LB_VAL;
+        if (f == LB_INC) done = true;
+        else q = qq + 1;
       }
-      st_relaxed_u64(st + tile * 256, LB_INC | (e + run));
+      if (done) break;
+      j -= q;
     }
-    s_gbase[t] = goff[t] + e;
+    st_relaxed_u64(st + tile * 256, LB_INC | (e + tcount));
   }
+  s_gbase[t] = goff[t] + e;
   __syncthreads();
 #pragma unroll
-  for (int i = 0; i < T_ITEMS; ++i)
-    if (d[i] < 256u) s_keys[s_lstart[d[i]] + s_whist[w][d[i]] + r[i]] = k[i];
+  for (int i = 0; i < T_ITEMS; ++i) {
+    uint32_t d = (uint32_t)(k[i] >> shift) & 255u;
+    if (full || wbase + i * 32 < n) s_keys[s_lstart[d] + s_whist[w][d] + r[i]] = k[i];
+  }
   __syncthreads();
   uint64_t valid_count = n - base < (uint64_t)T_TILE ? n - base : (uint64_t)T_TILE;
   for (uint32_t j = t; j < valid_count; j += T_THREADS) {

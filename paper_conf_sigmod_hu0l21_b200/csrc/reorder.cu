@@ -77,7 +77,15 @@ void build_oriented_csr(Graph &g) {
     TC_LAUNCH_CHECK();
   }
   uint64_t *sorted = keys.get();
-  if (!(ident && g.direct_rule == TC_DIRECT_ID)) {  // ID order + identity: already sorted
+  if (ident && g.direct_rule == TC_DIRECT_ID) {
+    // ID order + identity labels: the edge array is already the sorted oriented list
+  } else if (ident) {
+    // Original labels: the keys are in (min, max) order.  For a source s, its reversed
+    // edges (t < s) precede its forward block (t > s) and each group is ascending in t, so a
+    // STABLE sort on the source bits alone yields ascending N+(s): b bits instead of 2b.
+    tmp.alloc(m ? m : 1, s);
+    sorted = radix_sort_u64(keys.get(), tmp.get(), m, b, 2 * b, s);
+  } else {
     tmp.alloc(m ? m : 1, s);
     sorted = radix_sort_u64(keys.get(), tmp.get(), m, 0, 2 * b, s);
   }
