@@ -68,6 +68,8 @@ def lib():
         L.orc_oriented_csr.argtypes = [p, u64, u32, p, p, p, p]
         L.orc_count_forward.argtypes = [u32, p, p, u32, u32, p]
         L.orc_count_forward.restype = u64
+        L.orc_local_triangles.argtypes = [p, p, u64, p, u32, u32, p]
+        L.orc_local_triangles.restype = i32
         _LIB = L
     return _LIB
 
@@ -174,6 +176,17 @@ def count_forward(offs, col, u_begin=0, u_end=None, per_vertex=False):
     col = col if len(col) else np.zeros(1, dtype=np.uint32)
     T = lib().orc_count_forward(n, _p(offs), _p(col), u_begin, u_end, _p(tv))
     return (int(T), tv[:n]) if per_vertex else int(T)
+
+
+def local_triangles(src, dst, vertices, max_deg=4096):
+    """t(v) = #edges among N(v), straight from raw samples; UINT64_MAX when
+    d(v) > max_deg.  For sampled full-size parity (no graph build)."""
+    src = np.ascontiguousarray(src, dtype=np.uint32)
+    dst = np.ascontiguousarray(dst, dtype=np.uint32)
+    vs = np.ascontiguousarray(vertices, dtype=np.uint32)
+    out = np.zeros(max(len(vs), 1), dtype=np.uint64)
+    lib().orc_local_triangles(_p(src), _p(dst), len(src), _p(vs), len(vs), max_deg, _p(out))
+    return out[: len(vs)]
 
 
 def cost_eq1(n, m, od):

@@ -471,6 +471,104 @@ void orc_oriented_csr(const uint64_t *edges, uint64_t m, uint32_t n, const uint8
 }
 
 /* ------------------------------------------------------------------------ */
+/* Local (per-vertex) triangle counts straight from raw samples, by definition: */
+/* t(v) = number of edges among the neighbours N(v) of v in the simple graph    */
+/* (P:15).  For full-size parity on sampled vertices; needs no graph build.     */
+/* ------------------------------------------------------------------------ */
+
+typedef struct {
+  uint64_t *slot; /* key + 1, 0 = empty */
+  uint64_t cap;
+} u64set;
+
+static uint64_t mix64(uint64_t x) {
+  x ^= x >> 33; x *= 0xff51afd7ed558ccdull; x ^= x >> 33; x *= 0xc4ceb9fe1a85ec53ull; x ^= x >> 33;
+  return x;
+}
+
+static void set_init(u64set *s, uint64_t want) {
+  uint64_t cap = 16;
+  while (cap < 2 * want + 16) cap <<= 1;
+  s->cap = cap;
+  s->slot = (uint64_t *)calloc(cap, sizeof(uint64_t));
+}
+
+static int set_has(const u64set *s, uint64_t k) {
+  uint64_t i = mix64(k) & (s->cap - 1);
+  while (s->slot[i]) {
+    if (s->slot[i] == k + 1) return 1;
+    i = (i + 1) & (s->cap - 1);
+  }
+  return 0;
+}
+
+static void set_add(u64set *s, uint64_t k) {
+  uint64_t i = mix64(k) & (s->cap - 1);
+  while (s->slot[i]) {
+    if (s->slot[i] == k + 1) return;
+    i = (i + 1) & (s->cap - 1);
+  }
+  s->slot[i] = k + 1;
+}
+
+/* vs[0..nv): sampled vertices (each with degree <= max_deg in the simple graph, else
+ * t = UINT64_MAX is reported).  Two passes over the raw samples. */
+int orc_local_triangles(const uint32_t *src, const uint32_t *dst, uint64_t M, const uint32_t *vs,
+                        uint32_t nv, uint32_t max_deg, uint64_t *t_out) {
+  u64set S, X, E;
+  set_init(&S, nv);
+  for (uint32_t i = 0; i < nv; ++i) set_add(&S, vs[i]);
+  /* pass 1: neighbour sets of the sampled vertices, as (v << 32 | w) pairs */
+  uint64_t np = 0, cap = 1024;
+  uint64_t *pairs = (uint64_t *)malloc(cap * sizeof(uint64_t));
+  for (uint64_t i = 0; i < M; ++i) {
+    uint32_t a = src[i], b = dst[i];
+    if (a == b) continue;
+    for (int side = 0; side < 2; ++side) {
+      uint32_t v = side ? b : a, w = side ? a : b;
+      if (!set_has(&S, v)) continue;
+      if (np == cap) { cap *= 2; pairs = (uint64_t *)realloc(pairs, cap * sizeof(uint64_t)); }
+      pairs[np++] = ((uint64_t)v << 32) | w;
+    }
+  }
+  qsort(pairs, np, sizeof(uint64_t), cmp_u64);
+  uint64_t k = 0;
+  for (uint64_t i = 0; i < np; ++i)
+    if (k == 0 || pairs[k - 1] != pairs[i]) pairs[k++] = pairs[i];
+  np = k;
+  set_init(&X, np);
+  for (uint64_t i = 0; i < np; ++i) set_add(&X, (uint32_t)pairs[i]);
+  /* pass 2: every edge with both ends in X = ∪ N(v) */
+  set_init(&E, 4 * np + 1024);
+  for (uint64_t i = 0; i < M; ++i) {
+    uint32_t a = src[i], b = dst[i];
+    if (a == b || !set_has(&X, a) || !set_has(&X, b)) continue;
+    set_add(&E, edge_key(a, b));
+  }
+  /* t(v) = Σ over pairs x < y in N(v) of [ {x,y} ∈ E ] */
+  for (uint32_t q = 0; q < nv; ++q) {
+    uint32_t v = vs[q];
+    /* N(v) is the run of pairs with high word v (pairs sorted) */
+    uint64_t lo = 0, hi = np;
+    while (lo < hi) {
+      uint64_t mid = lo + (hi - lo) / 2;
+      if ((pairs[mid] >> 32) < v) lo = mid + 1;
+      else hi = mid;
+    }
+    uint64_t e = lo;
+    while (e < np && (pairs[e] >> 32) == v) ++e;
+    if (e - lo > max_deg) { t_out[q] = UINT64_MAX; continue; }
+    uint64_t t = 0;
+    for (uint64_t i = lo; i < e; ++i)
+      for (uint64_t j = i + 1; j < e; ++j)
+        t += set_has(&E, edge_key((uint32_t)pairs[i], (uint32_t)pairs[j]));
+    t_out[q] = t;
+  }
+  free(pairs); free(S.slot); free(X.slot); free(E.slot);
+  return 0;
+}
+
+/* ------------------------------------------------------------------------ */
 /* O4: count (forward algorithm): every triangle of the undirected graph */
 /* is counted once at its unique source u with u->v, u->w, v->w.       */
 /* ------------------------------------------------------------------------ */

@@ -34,32 +34,80 @@ static int64_t memory_superiority(uint32_t d, const tc_aorder_params &p) {
 }
 
 namespace {
+// Tournament (segment) tree over the buckets.  Each node stores its winner's key inline,
+// so an update touches only the leaf-to-root path (no indirection into mem_sup):
+// key = (+mem_sup, index) for the min queue, (-mem_sup, index) for the max queue, the
+// lexicographic minimum wins; a full bucket holds the +inf key.
 struct Tournament {
-  // node holds the winning leaf (bucket index) or -1; leaves beyond b are empty
-  std::vector<int64_t> node;
+  struct Node {
+    int64_t key;
+    uint32_t idx;
+  };
+  std::vector<Node> node;
   size_t P = 1;
-  const std::vector<int64_t> *sup = nullptr;
   bool want_max = false;
-  bool better(int64_t a, int64_t b) const {
-    if (a < 0) return false;
-    if (b < 0) return true;
-    int64_t x = (*sup)[a], y = (*sup)[b];
-    if (x != y) return want_max ? x > y : x < y;
-    return a < b;
+  static bool less(const Node &a, const Node &b) { return a.key != b.key ? a.key < b.key : a.idx < b.idx; }
+  Node leaf(size_t i, int64_t sup, bool alive) const {
+    if (!alive) return Node{INT64_MAX, UINT32_MAX};
+    return Node{want_max ? -sup : sup, (uint32_t)i};
   }
-  void build(size_t b, const std::vector<uint8_t> &alive) {
+  void build(size_t b, const std::vector<int64_t> &sup, const std::vector<uint8_t> &alive) {
     P = 1;
     while (P < b) P <<= 1;
-    node.assign(2 * P, -1);
-    for (size_t i = 0; i < b; ++i) node[P + i] = alive[i] ? (int64_t)i : -1;
-    for (size_t i = P - 1; i >= 1; --i) node[i] = better(node[2 * i], node[2 * i + 1]) ? node[2 * i] : node[2 * i + 1];
+    node.assign(2 * P, Node{INT64_MAX, UINT32_MAX});
+    for (size_t i = 0; i < b; ++i) node[P + i] = leaf(i, sup[i], alive[i]);
+    for (size_t i = P - 1; i >= 1; --i) node[i] = less(node[2 * i + 1], node[2 * i]) ? node[2 * i + 1] : node[2 * i];
   }
-  void update(size_t leaf, bool alive) {
-    size_t i = P + leaf;
-    node[i] = alive ? (int64_t)leaf : -1;
-    for (i >>= 1; i >= 1; i >>= 1) node[i] = better(node[2 * i], node[2 * i + 1]) ? node[2 * i] : node[2 * i + 1];
+  void update(size_t i, int64_t sup, bool alive) {
+    size_t x = P + i;
+    node[x] = leaf(i, sup, alive);
+    for (x >>= 1; x >= 1; x >>= 1) node[x] = less(node[2 * x + 1], node[2 * x]) ? node[2 * x + 1] : node[2 * x];
   }
-  int64_t top() const { return node[1]; }
+  int64_t top() const { return node[1].idx == UINT32_MAX ? -1 : (int64_t)node[1].idx; }
+};
+
+// Faster variant when (value, index) packs into 63 bits: one u64 per node (branchless min),
+// 4-ary heap layout (half the levels, children in one 32-B run).
+struct PackedTournament4 {
+  std::vector<uint64_t> node;  // internal nodes [0, nint), leaves [nint, nint + P)
+  size_t nint = 0, P = 1;
+  int ib = 1;          // index bits
+  int64_t off = 0;     // value offset making keys non-negative
+  bool want_max = false;
+  uint64_t pack(size_t i, int64_t sup, bool alive) const {
+    if (!alive) return UINT64_MAX;
+    int64_t v = want_max ? -sup : sup;
+    return ((uint64_t)(v + off) << ib) | (uint64_t)i;
+  }
+  void build(size_t b, const std::vector<int64_t> &sup, const std::vector<uint8_t> &alive) {
+    P = 1;
+    nint = 0;
+    while (P < b) {
+      nint += P;
+      P <<= 2;
+    }
+    node.assign(nint + P, UINT64_MAX);
+    for (size_t i = 0; i < b; ++i) node[nint + i] = pack(i, sup[i], alive[i]);
+    for (size_t x = nint; x-- > 0;) node[x] = min4(x);
+  }
+  uint64_t min4(size_t x) const {
+    const uint64_t *c = &node[4 * x + 1];
+    uint64_t a = c[0] < c[1] ? c[0] : c[1];
+    uint64_t b = c[2] < c[3] ? c[2] : c[3];
+    return a < b ? a : b;
+  }
+  void update(size_t i, int64_t sup, bool alive) {
+    size_t x = nint + i;
+    node[x] = pack(i, sup, alive);
+    while (x > 0) {
+      x = (x - 1) >> 2;
+      node[x] = min4(x);
+    }
+  }
+  int64_t top() const {
+    uint64_t t = node[0];
+    return t == UINT64_MAX ? -1 : (int64_t)(t & ((1ull << ib) - 1));
+  }
 };
 }  // namespace
 
@@ -101,26 +149,43 @@ void aorder_host(const std::vector<uint32_t> &od, const tc_aorder_params &p, std
   std::vector<uint32_t> fill(b, 0);
   std::vector<uint32_t> members(b * (size_t)k);
   std::vector<uint8_t> alive(b, 1);
-  Tournament q;
-  q.sup = &mem_sup;
-  if (b) {
+  // Phase 1 / phase 2 priority queues.  Packed 4-ary tree when max|mem_sup| and the bucket
+  // index fit 63 bits (always for the default parameters), else the generic tree.
+  int64_t smax = 0;
+  for (uint32_t v : vmem) smax = std::max<int64_t>(smax, std::llabs(S(od[v])));
+  for (uint32_t v : vcomp) smax = std::max<int64_t>(smax, std::llabs(S(od[v])));
+  const int ib = b > 1 ? 64 - __builtin_clzll((unsigned long long)(b - 1)) : 1;
+  const long double bound = (long double)smax * (long double)k * 2.0L + 2.0L;  // |mem_sup| < k smax
+  const bool packed = bound * (long double)(1ull << ib) < 9.0e18L;
+  auto run = [&](auto &q) {
     q.want_max = false;                      // line 2: min queue
-    q.build(b, alive);
+    q.build(b, mem_sup, alive);
     for (uint32_t v : vmem) {                // line 5
       int64_t bk = q.top();                  // line 6
       members[(size_t)bk * k + fill[bk]++] = v;  // line 7
       mem_sup[bk] += S(od[v]);               // line 8
       if (fill[bk] == k) alive[bk] = 0;
-      q.update((size_t)bk, alive[bk]);       // line 9
+      q.update((size_t)bk, mem_sup[bk], alive[bk]);  // line 9
     }
     q.want_max = true;                       // line 10: max queue
-    q.build(b, alive);
+    q.build(b, mem_sup, alive);
     for (uint32_t v : vcomp) {               // line 11
       int64_t bk = q.top();                  // line 12
       members[(size_t)bk * k + fill[bk]++] = v;  // line 13
       mem_sup[bk] += S(od[v]);               // line 14
       if (fill[bk] == k) alive[bk] = 0;
-      q.update((size_t)bk, alive[bk]);       // line 15
+      q.update((size_t)bk, mem_sup[bk], alive[bk]);  // line 15
+    }
+  };
+  if (b) {
+    if (packed) {
+      PackedTournament4 q;
+      q.ib = ib;
+      q.off = (int64_t)(smax * (int64_t)k + 1);
+      run(q);
+    } else {
+      Tournament q;
+      run(q);
     }
   }
   perm.assign(n, 0);

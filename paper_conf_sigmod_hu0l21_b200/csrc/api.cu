@@ -421,7 +421,10 @@ tc_status tc_analyze(tc_graph *gp) {
 tc_status tc_get_stats(const tc_graph *gp, tc_stats_t *o) {
   return guard([&] {
     TC_REQUIRE(gp && o, ST_INVALID, "NULL argument");
-    const Graph &g = *gp;
+    Graph &g = *const_cast<tc_graph *>(gp);  // lazily filled statistics (no logical change)
+    TC_CUDA(cudaSetDevice(g.device));
+    ensure_max_degree(g);
+    if (g.state >= G_DIRECTED) ensure_od(g);
     std::memset(o, 0, sizeof(*o));
     o->n = g.n;
     o->m = g.m;
@@ -495,6 +498,7 @@ tc_status tc_export_direct(tc_graph *gp, uint32_t *outdeg, uint32_t *sub, uint32
   return guard([&] {
     Graph &g = checked(gp, G_DIRECTED);
     TC_REQUIRE(!(sub || dsnap) || g.direct_rule == TC_DIRECT_PAPER, ST_STATE, "sub/dsnap exist only for PAPER");
+    if (outdeg) ensure_od(g);
     copy_out(outdeg, g.od.get(), 4ull * g.n, g.stream);
     copy_out(sub, g.sub.get(), 4ull * g.n, g.stream);
     copy_out(dsnap, g.dsnap.get(), 4ull * g.n, g.stream);

@@ -2,54 +2,21 @@
 //
 //   canonicalize : key = (min(u,v) << b) | max(u,v), b = bits(n-1); a self-loop maps to the
 //                  all-ones sentinel (it cannot be an edge key since u < v) so no compaction
-//                  pass is needed; ids >= n raise an error flag (TC_ERR_INVALID).
+//                  pass is needed; ids >= n raise an error flag (TC_ERR_INVALID).  Fused into
+//                  the radix sort's histogram and first pass (no key array is materialised).
 //   radix sort   : 2b significant bits (prims.cu)
-//   unique       : first key of every run (duplicates and both directions merged, Q1)
-//   degrees      : d(v) via warp-aggregated atomics
+//   unique       : first key of every run (duplicates and both directions merged, Q1),
+//                  fused with the degrees d(v) (run-aggregated atomics)
 #include "internal.h"
 #include "prims.cuh"
 
 namespace tc {
 namespace {
 
-__global__ void canonicalize_kernel(const uint32_t *__restrict__ src, const uint32_t *__restrict__ dst,
-                                    uint64_t M, uint32_t n, int bits, uint64_t sentinel,
-                                    uint64_t *__restrict__ keys, unsigned *err) {
-  uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < M; i += stride) {
-    uint32_t u = src[i], v = dst[i];
-    if (u >= n || v >= n) {
-      atomicOr(err, 1u);
-      keys[i] = sentinel;
-      continue;
-    }
-    uint32_t lo = min(u, v), hi = max(u, v);
-    keys[i] = (u == v) ? sentinel : (((uint64_t)lo << bits) | hi);
-  }
-}
-
 // m = runs - (last run is the sentinel)
 __global__ void trim_sentinel_kernel(const uint64_t *uniq, uint64_t *d_count, uint64_t sentinel) {
   uint64_t c = *d_count;
   if (c > 0 && uniq[c - 1] == sentinel) *d_count = c - 1;
-}
-
-__global__ void degree_kernel(const uint64_t *__restrict__ edges, uint64_t m, int bits,
-                              uint32_t *__restrict__ deg) {
-  uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-  uint64_t mask = (1ull << bits) - 1;
-  // warp-uniform loop so __match_any_sync sees full warps
-  for (uint64_t base = (uint64_t)blockIdx.x * blockDim.x + (threadIdx.x & ~31u); base < m; base += stride) {
-    uint64_t i = base + lane_id();
-    bool valid = i < m;
-    uint64_t k = valid ? edges[i] : 0;
-    uint32_t u = valid ? (uint32_t)(k >> bits) : 0xffffffffu;
-    uint32_t v = (uint32_t)(k & mask);
-    // sorted keys: runs of equal u are contiguous -> aggregate them
-    unsigned peers = __match_any_sync(0xffffffffu, u);
-    if (valid && lane_id() == (unsigned)(__ffs(peers) - 1)) atomicAdd(&deg[u], (uint32_t)__popc(peers));
-    if (valid) atomicAdd(&deg[v], 1u);
-  }
 }
 
 __global__ void max_kernel(const uint32_t *__restrict__ a, uint64_t n, unsigned *out) {
@@ -93,15 +60,13 @@ void build_graph(Graph &g, const uint32_t *d_src, const uint32_t *d_dst, uint64_
   DevBuf<uint64_t> d_m;
   d_m.alloc(1, s);
   TC_CUDA(cudaMemsetAsync(err.get(), 0, sizeof(unsigned), s));
-  if (M) {
-    ProfScope prof("canonicalize", s, 16.0 * M);
-    canonicalize_kernel<<<grid_for(M, 256), 256, 0, s>>>(d_src, d_dst, M, n, b, sentinel, keys.get(),
-                                                          err.get());
-    TC_LAUNCH_CHECK();
-  }
-  uint64_t *sorted = radix_sort_u64(keys.get(), tmp.get(), M, 0, 2 * b, s);
+  g.deg.alloc(n ? n : 1, s);
+  TC_CUDA(cudaMemsetAsync(g.deg.get(), 0, g.deg.bytes(), s));
+  // a1+a2: canonicalise inside the radix sort's histogram and first pass
+  uint64_t *sorted = radix_sort_edges(d_src, d_dst, M, n, b, sentinel, keys.get(), tmp.get(), err.get(), s);
   uint64_t *uniq = (sorted == keys.get()) ? tmp.get() : keys.get();
-  unique_sorted_u64(sorted, uniq, M, d_m.get(), s);
+  // a2+a3: unique runs and undirected degrees in one pass
+  unique_sorted_u64(sorted, uniq, M, d_m.get(), s, g.deg.get(), b, sentinel);
   trim_sentinel_kernel<<<1, 1, 0, s>>>(uniq, d_m.get(), sentinel);
   TC_LAUNCH_CHECK();
   unsigned h_err = 0;
@@ -114,16 +79,14 @@ void build_graph(Graph &g, const uint32_t *d_src, const uint32_t *d_dst, uint64_
   // keep the unique run as the edge array; release the other buffer
   if (uniq == keys.get()) g.edges = std::move(keys);
   else g.edges = std::move(tmp);
-
-  g.deg.alloc(n ? n : 1, s);
-  TC_CUDA(cudaMemsetAsync(g.deg.get(), 0, g.deg.bytes(), s));
-  if (g.m) {
-    ProfScope prof("degree", s, 8.0 * g.m + 8.0 * g.m);
-    degree_kernel<<<grid_for(g.m, 256), 256, 0, s>>>(g.edges.get(), g.m, b, g.deg.get());
-    TC_LAUNCH_CHECK();
-  }
-  g.max_degree = device_max_u32(g.deg.get(), n, s);
+  g.max_degree_ready = false;
   g.state = G_BUILT;
+}
+
+void ensure_max_degree(Graph &g) {
+  if (g.max_degree_ready) return;
+  g.max_degree = device_max_u32(g.deg.get(), g.n, g.stream);
+  g.max_degree_ready = true;
 }
 
 }  // namespace tc

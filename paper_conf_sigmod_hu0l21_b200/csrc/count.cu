@@ -46,6 +46,10 @@ struct WarpScratch {  // per-warp owner-search tables for one 32-v chunk
 
 __device__ __forceinline__ uint32_t ldg_u32(const uint32_t *p) { return __ldg(p); }
 
+// Dynamic shared memory of every count kernel.  Searches index it directly so the
+// compiler emits 32-bit LDS (not generic loads) for the binary-search steps.
+extern __shared__ __align__(128) uint32_t tc_smem[];
+
 // Branchless search: does `w` occur in the ascending list s[0..L), L >= 1? (any memory)
 __device__ __forceinline__ bool bsearch_list(const uint32_t *s, uint32_t L, uint32_t w) {
   const uint32_t *p = s;
@@ -62,14 +66,14 @@ __device__ __forceinline__ bool bsearch_list(const uint32_t *s, uint32_t L, uint
 // entries: S unrolled steps of one shared load + compare + select each ("binary lifting").
 // Precondition: s[0] <= w (the caller's range filter).
 template <int S>
-__device__ __forceinline__ bool bsearch_pow2(const uint32_t *s, uint32_t w) {
-  uint32_t p = 0;
+__device__ __forceinline__ bool bsearch_pow2(uint32_t sbase, uint32_t w) {
+  uint32_t p = sbase;
 #pragma unroll
   for (int k = S - 1; k >= 0; --k) {
     uint32_t q = p + (1u << k);
-    p = (s[q] <= w) ? q : p;
+    p = (tc_smem[q] <= w) ? q : p;
   }
-  return s[p] == w;
+  return tc_smem[p] == w;
 }
 
 __device__ __forceinline__ int ceil_log2(uint32_t L) { return L <= 1 ? 0 : 32 - __clz(L - 1); }
@@ -79,31 +83,47 @@ __device__ __forceinline__ int ceil_log2(uint32_t L) { return L <= 1 ? 0 : 32 - 
 // incrementally (its wedge index grows by 32 per step), so locating w's list costs ~1
 // shared load per wedge instead of a 5-step search.
 template <bool PV, int S>
-__device__ __forceinline__ uint32_t wedge_loop(const uint32_t *__restrict__ col, const uint32_t *list, uint32_t L,
-                                               uint32_t lo, uint32_t hi, uint32_t total, const WarpScratch &ws,
-                                               unsigned long long *tv) {
+__device__ __forceinline__ uint32_t wedge_loop(const uint32_t *__restrict__ col, const uint32_t *list, uint32_t sbase,
+                                               uint32_t L, uint32_t lo, uint32_t hi, uint32_t total,
+                                               const WarpScratch &ws, unsigned long long *tv) {
   uint32_t cnt = 0;
   uint32_t o = 0, o_beg = 0, o_end = ws.pre[0];
   uint64_t o_vb = ws.vb[0];
-  for (uint32_t j = lane_id(); j < total; j += 32) {
-    if (o_end <= j) {
-      do {
-        ++o;
-        o_beg = o_end;
-        o_end = ws.pre[o];
-      } while (o_end <= j);
-      o_vb = ws.vb[o];
+  // UNR wedges per lane in flight: their loads are issued back to back before any search
+  // (memory-level parallelism for the gather; the owner walk stays incremental).
+  constexpr int UNR = 4;
+  for (uint32_t j0 = lane_id(); j0 < total; j0 += 32 * UNR) {
+    uint32_t w[UNR], ow[UNR];
+#pragma unroll
+    for (int k = 0; k < UNR; ++k) {
+      const uint32_t j = j0 + 32 * k;
+      w[k] = 0xffffffffu;  // > hi: filtered out
+      ow[k] = o;
+      if (j < total) {
+        if (o_end <= j) {
+          do {
+            ++o;
+            o_beg = o_end;
+            o_end = ws.pre[o];
+          } while (o_end <= j);
+          o_vb = ws.vb[o];
+        }
+        ow[k] = o;
+        w[k] = ldg_u32(col + o_vb + (j - o_beg));
+      }
     }
-    const uint32_t w = ldg_u32(col + o_vb + (j - o_beg));
-    if (w >= lo && w <= hi) {
-      bool hit;
-      if (S > 0) hit = bsearch_pow2<S>(list, w);
-      else hit = bsearch_list(list, L, w);
-      if (hit) {
-        ++cnt;
-        if (PV) {
-          atomicAdd(&tv[w], 1ull);
-          atomicAdd(&tv[ws.v[o]], 1ull);
+#pragma unroll
+    for (int k = 0; k < UNR; ++k) {
+      if (w[k] >= lo && w[k] <= hi) {
+        bool hit;
+        if (S > 0) hit = bsearch_pow2<S>(sbase, w[k]);
+        else hit = bsearch_list(list, L, w[k]);
+        if (hit) {
+          ++cnt;
+          if (PV) {
+            atomicAdd(&tv[w[k]], 1ull);
+            atomicAdd(&tv[ws.v[ow[k]]], 1ull);
+          }
         }
       }
     }
@@ -112,12 +132,13 @@ __device__ __forceinline__ uint32_t wedge_loop(const uint32_t *__restrict__ col,
 }
 
 // Count the wedges u->v->w of one chunk of up to 32 v's (lane-held `v`, `valid`) whose w
-// lies in list[0..L) (w restricted to [lo, hi]).  `padded`: list is padded with +inf to
-// 2^ceil(log2 L) entries (shared-memory copies).  Returns this lane's matches.
+// lies in list[0..L) (w restricted to [lo, hi]).  `padded`: list is the shared-memory copy
+// tc_smem[sbase ..] padded with +inf to 2^ceil(log2 L) entries.  Returns this lane's matches.
 template <bool PV>
 __device__ __forceinline__ uint32_t warp_chunk(const uint64_t *__restrict__ offs, const uint32_t *__restrict__ col,
-                                               uint32_t v, bool valid, const uint32_t *list, uint32_t L, bool padded,
-                                               uint32_t lo, uint32_t hi, WarpScratch &ws, unsigned long long *tv) {
+                                               uint32_t v, bool valid, const uint32_t *list, uint32_t sbase,
+                                               uint32_t L, bool padded, uint32_t lo, uint32_t hi, WarpScratch &ws,
+                                               unsigned long long *tv) {
   const unsigned lane = lane_id();
   uint64_t vb = 0;
   uint32_t dv = 0;
@@ -141,13 +162,13 @@ __device__ __forceinline__ uint32_t warp_chunk(const uint64_t *__restrict__ offs
     switch (S) {
 #define TC_CASE(k) \
   case k:          \
-    cnt = wedge_loop<PV, k>(col, list, L, lo, hi, total, ws, tv); \
+    cnt = wedge_loop<PV, k>(col, list, sbase, L, lo, hi, total, ws, tv); \
     break;
       TC_CASE(1) TC_CASE(2) TC_CASE(3) TC_CASE(4) TC_CASE(5) TC_CASE(6) TC_CASE(7)
       TC_CASE(8) TC_CASE(9) TC_CASE(10) TC_CASE(11) TC_CASE(12) TC_CASE(13) TC_CASE(14)
 #undef TC_CASE
       default:
-        cnt = wedge_loop<PV, 0>(col, list, L, lo, hi, total, ws, tv);
+        cnt = wedge_loop<PV, 0>(col, list, sbase, L, lo, hi, total, ws, tv);
     }
   }
   __syncwarp();
@@ -159,7 +180,7 @@ __device__ __forceinline__ uint32_t warp_chunk(const uint64_t *__restrict__ offs
 // else in global memory.
 template <bool PV>
 __device__ __forceinline__ uint64_t warp_item(const uint64_t *__restrict__ offs, const uint32_t *__restrict__ col,
-                                              uint32_t u, uint32_t c0, uint32_t *slice, uint32_t cap,
+                                              uint32_t u, uint32_t c0, uint32_t sbase, uint32_t cap,
                                               WarpScratch &ws, unsigned long long *tv) {
   const unsigned lane = lane_id();
   const uint64_t a = offs[u];
@@ -169,9 +190,9 @@ __device__ __forceinline__ uint64_t warp_item(const uint64_t *__restrict__ offs,
   bool padded = false;
   if (L <= cap) {
     const uint32_t P = 1u << ceil_log2(L);
-    for (uint32_t j = lane; j < P; j += 32) slice[j] = j < L ? ldg_u32(col + a + j) : 0xffffffffu;
+    for (uint32_t j = lane; j < P; j += 32) tc_smem[sbase + j] = j < L ? ldg_u32(col + a + j) : 0xffffffffu;
     __syncwarp();
-    list = slice;
+    list = tc_smem + sbase;
     padded = true;
   } else {
     list = col + a;
@@ -179,7 +200,7 @@ __device__ __forceinline__ uint64_t warp_item(const uint64_t *__restrict__ offs,
   const uint32_t lo = list[0], hi = list[L - 1];
   const bool valid = c0 + lane < L;
   const uint32_t v = valid ? list[c0 + lane] : 0u;
-  uint32_t cnt = warp_chunk<PV>(offs, col, v, valid, list, L, padded, lo, hi, ws, tv);
+  uint32_t cnt = warp_chunk<PV>(offs, col, v, valid, list, sbase, L, padded, lo, hi, ws, tv);
   __syncwarp();  // slice reads done before the next item restages it
   if (PV) {
     uint64_t tot = warp_sum((uint64_t)cnt);
@@ -281,9 +302,8 @@ __global__ __launch_bounds__(CT_THREADS) void count_small_kernel(const uint64_t 
                                                                  const uint64_t *__restrict__ items, uint64_t nitems,
                                                                  uint64_t nheavy, unsigned long long *ctr, uint32_t cap,
                                                                  unsigned long long *T, unsigned long long *tv) {
-  extern __shared__ uint32_t s_dyn[];
   __shared__ WarpScratch s_ws[CT_WARPS];
-  uint32_t *slice = s_dyn + warp_id() * cap;
+  const uint32_t slice = warp_id() * cap;
   WarpScratch &ws = s_ws[warp_id()];
   uint64_t acc = 0;
   while (true) {  // heavy items, one per fetch
@@ -345,7 +365,7 @@ __global__ __launch_bounds__(LG_THREADS) void count_large_kernel(const uint64_t 
                                                                  const uint64_t *__restrict__ items, uint64_t nitems,
                                                                  unsigned long long *ctr, unsigned long long *T,
                                                                  unsigned long long *tv) {
-  extern __shared__ __align__(128) uint32_t s_piece[];  // PIECE + 8 words (alignment slack)
+  uint32_t *s_piece = tc_smem;  // PIECE + 8 words (alignment slack)
   __shared__ WarpScratch s_ws[LG_WARPS];
   __shared__ __align__(8) uint64_t s_bar;
   __shared__ unsigned long long s_item;
@@ -392,7 +412,7 @@ __global__ __launch_bounds__(LG_THREADS) void count_large_kernel(const uint64_t 
       for (uint32_t c0 = cbeg + warp_id() * 32; c0 < cend; c0 += LG_THREADS) {
         bool valid = c0 + lane_id() < cend;
         uint32_t v = valid ? ldg_u32(col + a + c0 + lane_id()) : 0u;
-        cnt += warp_chunk<PV>(offs, col, v, valid, list, plen, true, lo, hi, ws, tv);
+        cnt += warp_chunk<PV>(offs, col, v, valid, list, shift, plen, true, lo, hi, ws, tv);
       }
       ucnt += cnt;
       __syncthreads();  // piece fully consumed before the next bulk copy overwrites it
@@ -414,9 +434,8 @@ __global__ __launch_bounds__(CT_THREADS) void count_range_kernel(const uint64_t 
                                                                  uint32_t b0, uint32_t nb, uint32_t ub, uint32_t ue,
                                                                  uint32_t cap, unsigned long long *T,
                                                                  unsigned long long *tv) {
-  extern __shared__ uint32_t s_dyn[];
   __shared__ WarpScratch s_ws[CT_WARPS];
-  uint32_t *slice = s_dyn + warp_id() * cap;
+  const uint32_t slice = warp_id() * cap;
   WarpScratch &ws = s_ws[warp_id()];
   uint64_t acc = 0;
   for (uint32_t bi = b0 + blockIdx.x; bi < b0 + nb; bi += gridDim.x) {

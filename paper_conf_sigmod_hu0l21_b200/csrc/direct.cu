@@ -23,7 +23,6 @@
 
 namespace tc {
 
-uint32_t device_max_u32(const uint32_t *a, uint64_t n, cudaStream_t s);
 
 namespace {
 
@@ -120,6 +119,14 @@ __global__ void outdeg_kernel(const uint64_t *__restrict__ edges, uint64_t m, in
     uint32_t u = (uint32_t)(k >> bits), v = (uint32_t)(k & mask);  // u < v
     uint32_t s = prim[u] <= prim[v] ? u : v;
     atomicAdd(&od[s], 1u);
+  }
+}
+
+__global__ void od_from_offs_kernel(const uint64_t *__restrict__ offs, const uint32_t *__restrict__ perm, uint32_t n,
+                                    uint32_t *__restrict__ od) {
+  for (uint64_t v = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (uint64_t)gridDim.x * blockDim.x) {
+    uint32_t p = perm ? perm[v] : (uint32_t)v;
+    od[v] = (uint32_t)(offs[p + 1] - offs[p]);
   }
 }
 
@@ -238,29 +245,8 @@ void direct_graph(Graph &g, int rule) {
   } else {
     peel_paper(g);
   }
-  g.od.alloc(n ? n : 1, s);
-  TC_CUDA(cudaMemsetAsync(g.od.get(), 0, g.od.bytes(), s));
-  if (g.m) {
-    ProfScope prof("outdeg", s, 8.0 * g.m + 16.0 * g.m);
-    outdeg_kernel<<<grid_for(g.m, 256), 256, 0, s>>>(g.edges.get(), g.m, g.bits, g.prim.get(), g.od.get());
-    TC_LAUNCH_CHECK();
-  }
-  g.max_outdeg = device_max_u32(g.od.get(), n, s);
-  // Eq.1 statistic (P:146-148)
-  {
-    unsigned blocks = grid_for(n, 256, 2);
-    DevBuf<unsigned long long> part;
-    part.alloc(2 * blocks, s);
-    eq1_kernel<<<blocks, 256, 0, s>>>(g.od.get(), n, g.m, part.get());
-    TC_LAUNCH_CHECK();
-    std::vector<unsigned long long> h(2 * blocks);
-    TC_CUDA(cudaMemcpyAsync(h.data(), part.get(), part.bytes(), cudaMemcpyDeviceToHost, s));
-    TC_CUDA(cudaStreamSynchronize(s));
-    unsigned __int128 t = 0;
-    for (unsigned i = 0; i < blocks; ++i) t += ((unsigned __int128)h[2 * i + 1] << 64) | h[2 * i];
-    g.eq1_lo = (uint64_t)t;
-    g.eq1_hi = (uint64_t)(t >> 64);
-  }
+  g.od.release();
+  g.od_ready = false;  // computed on demand (ensure_od): not needed by NONE ordering
   g.direct_rule = rule;
   g.reorder_rule = -1;
   g.identity_perm = true;
@@ -272,6 +258,42 @@ void direct_graph(Graph &g, int rule) {
   g.col.release();
   g.csr_ready = false;
   g.state = G_DIRECTED;
+}
+
+void ensure_od(Graph &g) {
+  if (g.od_ready) return;
+  cudaStream_t s = g.stream;
+  const uint32_t n = g.n;
+  g.od.alloc(n ? n : 1, s);
+  if (g.csr_ready) {  // d~ = list lengths of the oriented CSR
+    if (n) {
+      od_from_offs_kernel<<<grid_for(n, 256), 256, 0, s>>>(g.offs.get(), g.identity_perm ? nullptr : g.perm.get(), n,
+                                                           g.od.get());
+      TC_LAUNCH_CHECK();
+    }
+  } else {
+    TC_CUDA(cudaMemsetAsync(g.od.get(), 0, g.od.bytes(), s));
+    if (g.m) {
+      ProfScope prof("outdeg", s, 8.0 * g.m + 16.0 * g.m);
+      outdeg_kernel<<<grid_for(g.m, 256), 256, 0, s>>>(g.edges.get(), g.m, g.bits, g.prim.get(), g.od.get());
+      TC_LAUNCH_CHECK();
+    }
+  }
+  g.max_outdeg = device_max_u32(g.od.get(), n, s);
+  // Eq.1 statistic (P:146-148)
+  unsigned blocks = grid_for(n, 256, 2);
+  DevBuf<unsigned long long> part;
+  part.alloc(2 * blocks, s);
+  eq1_kernel<<<blocks, 256, 0, s>>>(g.od.get(), n, g.m, part.get());
+  TC_LAUNCH_CHECK();
+  std::vector<unsigned long long> h(2 * blocks);
+  TC_CUDA(cudaMemcpyAsync(h.data(), part.get(), part.bytes(), cudaMemcpyDeviceToHost, s));
+  TC_CUDA(cudaStreamSynchronize(s));
+  unsigned __int128 t = 0;
+  for (unsigned i = 0; i < blocks; ++i) t += ((unsigned __int128)h[2 * i + 1] << 64) | h[2 * i];
+  g.eq1_lo = (uint64_t)t;
+  g.eq1_hi = (uint64_t)(t >> 64);
+  g.od_ready = true;
 }
 
 }  // namespace tc

@@ -25,6 +25,8 @@ struct Graph {
   DevBuf<uint64_t> edges;  // m packed keys (u << bits) | v, u < v, ascending
   DevBuf<uint32_t> deg;    // d(v)
   uint32_t max_degree = 0;
+  bool max_degree_ready = false;
+  bool od_ready = false;  // od / max_outdeg / eq1 are computed lazily (ensure_od)
 
   // a4-a5: directing
   int direct_rule = -1;
@@ -56,8 +58,11 @@ struct Graph {
 
 // build.cu
 void build_graph(Graph &g, const uint32_t *d_src, const uint32_t *d_dst, uint64_t M);
+void ensure_max_degree(Graph &g);
+uint32_t device_max_u32(const uint32_t *a, uint64_t n, cudaStream_t s);
 // direct.cu
 void direct_graph(Graph &g, int rule);
+void ensure_od(Graph &g);  // out-degrees d~ (original ids), max d~, Eq.1 numerator
 // reorder.cu
 void reorder_graph(Graph &g, int rule, const tc_aorder_params &p);
 void build_oriented_csr(Graph &g);

@@ -18,6 +18,32 @@ constexpr int T_TILE = T_THREADS * T_ITEMS;  // 4096
 constexpr int T_WARPS = T_THREADS / 32;
 constexpr int MAX_PASSES = 8;
 
+// ------------------------------------------------------------------ key sources
+// Radix-sort input loaders: plain keys, or raw edge samples canonicalised on the fly
+// (step a1 fused into the histogram and the first pass: (min << b) | max, self-loop or
+// out-of-range id -> all-ones sentinel; out-of-range ids also raise *err).
+struct KeySrc {
+  const uint64_t *__restrict__ k;
+  __device__ __forceinline__ uint64_t load(uint64_t i) const { return __ldcs(k + i); }
+};
+struct EdgeSrc {
+  const uint32_t *__restrict__ src;
+  const uint32_t *__restrict__ dst;
+  uint32_t n;
+  int bits;
+  uint64_t sentinel;
+  unsigned *err;  // set only by the histogram kernel
+  __device__ __forceinline__ uint64_t load(uint64_t i) const {
+    uint32_t u = __ldcs(src + i), v = __ldcs(dst + i);
+    if (u >= n || v >= n) {
+      if (err) atomicOr(err, 1u);
+      return sentinel;
+    }
+    if (u == v) return sentinel;
+    return ((uint64_t)min(u, v) << bits) | max(u, v);
+  }
+};
+
 // ------------------------------------------------------------------ scan
 template <typename TI>
 __global__ __launch_bounds__(T_THREADS) void scan_kernel(const TI *__restrict__ in,
@@ -52,10 +78,13 @@ __global__ __launch_bounds__(T_THREADS) void scan_kernel(const TI *__restrict__ 
 }
 
 // ------------------------------------------------------------------ unique
+// Unique-select; optionally (deg != nullptr) the undirected degrees of the kept edges
+// (step a3 fused): keys are (u << bits) | v, u < v; the sentinel key is dropped from deg.
 __global__ __launch_bounds__(T_THREADS) void unique_kernel(const uint64_t *__restrict__ in,
                                                            uint64_t *__restrict__ out, uint64_t n,
                                                            uint64_t *status, uint32_t *tile_ctr,
-                                                           uint64_t ntiles, uint64_t *d_count) {
+                                                           uint64_t ntiles, uint64_t *d_count, uint32_t *deg,
+                                                           int bits, uint64_t sentinel) {
   __shared__ uint64_t s_warp[8];
   __shared__ uint64_t s_total;
   __shared__ uint32_t s_tile;
@@ -86,12 +115,29 @@ __global__ __launch_bounds__(T_THREADS) void unique_kernel(const uint64_t *__res
 #pragma unroll
   for (int i = 0; i < T_ITEMS; ++i)
     if (flags >> i & 1u) out[pos++] = k[i];
+  if (deg) {
+    const uint64_t mask = (1ull << bits) - 1;
+    uint32_t ru = 0xffffffffu, rc = 0;  // run of equal u among this thread's heads
+#pragma unroll
+    for (int i = 0; i < T_ITEMS; ++i) {
+      if (!(flags >> i & 1u) || k[i] == sentinel) continue;
+      uint32_t u = (uint32_t)(k[i] >> bits), v = (uint32_t)(k[i] & mask);
+      atomicAdd(&deg[v], 1u);
+      if (u != ru) {
+        if (rc) atomicAdd(&deg[ru], rc);
+        ru = u;
+        rc = 0;
+      }
+      ++rc;
+    }
+    if (rc) atomicAdd(&deg[ru], rc);
+  }
 }
 
 // ------------------------------------------------------------------ radix sort
 // Up-front digit histograms for every pass; per-warp private smem counters.
-__global__ __launch_bounds__(T_THREADS) void rs_hist_kernel(const uint64_t *__restrict__ keys,
-                                                            uint64_t n, int begin_bit, int passes,
+template <class Src>
+__global__ __launch_bounds__(T_THREADS) void rs_hist_kernel(Src keys, uint64_t n, int begin_bit, int passes,
                                                             unsigned long long *ghist) {
   extern __shared__ uint32_t s_h[];  // [T_WARPS/2][passes][256]
   const int groups = T_WARPS / 2;
@@ -100,7 +146,7 @@ __global__ __launch_bounds__(T_THREADS) void rs_hist_kernel(const uint64_t *__re
   uint32_t *mine = s_h + (warp_id() / 2) * passes * 256;
   uint64_t stride = (uint64_t)gridDim.x * T_THREADS;
   for (uint64_t i = (uint64_t)blockIdx.x * T_THREADS + threadIdx.x; i < n; i += stride) {
-    uint64_t k = keys[i];
+    uint64_t k = keys.load(i);
     for (int p = 0; p < passes; ++p) atomicAdd(&mine[p * 256 + ((k >> (begin_bit + 8 * p)) & 255u)], 1u);
   }
   __syncthreads();
@@ -145,8 +191,8 @@ __device__ __forceinline__ uint32_t rank_item(uint32_t d, bool valid, uint32_t *
   return old + __popc(peers & lt_mask);
 }
 
-__global__ __launch_bounds__(T_THREADS, 3) void rs_pass_kernel(const uint64_t *__restrict__ in,
-                                                               uint64_t *__restrict__ out, uint64_t n,
+template <class Src>
+__global__ __launch_bounds__(T_THREADS, 3) void rs_pass_kernel(Src in, uint64_t *__restrict__ out, uint64_t n,
                                                                int shift,
                                                                const unsigned long long *__restrict__ goff,
                                                                uint64_t *status, uint32_t *tile_ctr) {
@@ -173,10 +219,10 @@ __global__ __launch_bounds__(T_THREADS, 3) void rs_pass_kernel(const uint64_t *_
   const uint64_t wbase = base + w * (32 * T_ITEMS) + l;  // warp-striped: stable order
   if (full) {
 #pragma unroll
-    for (int i = 0; i < T_ITEMS; ++i) k[i] = __ldcs(in + wbase + i * 32);
+    for (int i = 0; i < T_ITEMS; ++i) k[i] = in.load(wbase + i * 32);
   } else {
 #pragma unroll
-    for (int i = 0; i < T_ITEMS; ++i) k[i] = (wbase + i * 32 < n) ? in[wbase + i * 32] : ~0ull;
+    for (int i = 0; i < T_ITEMS; ++i) k[i] = (wbase + i * 32 < n) ? in.load(wbase + i * 32) : ~0ull;
   }
   // early tile histogram -> publish the aggregate before the (long) ranking so that
   // successors' look-back rarely waits (one-sweep "early counts")
@@ -270,8 +316,8 @@ void scan_u64(const uint64_t *in, uint64_t *out, uint64_t n, cudaStream_t s) {
   scan_impl<uint64_t>(in, out, n, s);
 }
 
-void unique_sorted_u64(const uint64_t *in, uint64_t *out, uint64_t n, uint64_t *d_count,
-                       cudaStream_t s) {
+void unique_sorted_u64(const uint64_t *in, uint64_t *out, uint64_t n, uint64_t *d_count, cudaStream_t s,
+                       uint32_t *deg, int bits, uint64_t sentinel) {
   if (n == 0) {
     TC_CUDA(cudaMemsetAsync(d_count, 0, sizeof(uint64_t), s));
     return;
@@ -281,16 +327,16 @@ void unique_sorted_u64(const uint64_t *in, uint64_t *out, uint64_t n, uint64_t *
   scratch.alloc(ntiles + 1, s);
   TC_CUDA(cudaMemsetAsync(scratch.get(), 0, scratch.bytes(), s));
   ProfScope prof("unique", s, 8.0 * n);
-  unique_kernel<<<(unsigned)ntiles, T_THREADS, 0, s>>>(in, out, n, scratch.get() + 1,
-                                                       (uint32_t *)scratch.get(), ntiles, d_count);
+  unique_kernel<<<(unsigned)ntiles, T_THREADS, 0, s>>>(in, out, n, scratch.get() + 1, (uint32_t *)scratch.get(),
+                                                       ntiles, d_count, deg, bits, sentinel);
   TC_LAUNCH_CHECK();
 }
 
-uint64_t *radix_sort_u64(uint64_t *keys, uint64_t *tmp, uint64_t n, int begin_bit, int end_bit,
-                         cudaStream_t s) {
-  if (n <= 1 || end_bit <= begin_bit) return keys;
+template <class Src>
+static uint64_t *radix_sort_impl(Src first, uint64_t *out0, uint64_t *out1, uint64_t n, int begin_bit, int end_bit,
+                                 cudaStream_t s) {
   int passes = (end_bit - begin_bit + 7) / 8;
-  TC_REQUIRE(passes <= MAX_PASSES, ST_INVALID, "radix sort: too many bits");
+  TC_REQUIRE(passes >= 1 && passes <= MAX_PASSES, ST_INVALID, "radix sort: bad bit range");
   uint64_t ntiles = (n + T_TILE - 1) / T_TILE;
   DevBuf<unsigned long long> hist;
   hist.alloc((size_t)passes * 256, s);
@@ -298,31 +344,48 @@ uint64_t *radix_sort_u64(uint64_t *keys, uint64_t *tmp, uint64_t n, int begin_bi
   size_t hsm = (size_t)(T_WARPS / 2) * passes * 256 * sizeof(uint32_t);
   static bool attr_set = false;
   if (!attr_set) {
-    TC_CUDA(cudaFuncSetAttribute(rs_hist_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                 (int)((T_WARPS / 2) * MAX_PASSES * 256 * sizeof(uint32_t))));
+    int mx = (int)((T_WARPS / 2) * MAX_PASSES * 256 * sizeof(uint32_t));
+    TC_CUDA(cudaFuncSetAttribute(rs_hist_kernel<KeySrc>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx));
+    TC_CUDA(cudaFuncSetAttribute(rs_hist_kernel<EdgeSrc>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx));
     attr_set = true;
   }
   {
     ProfScope prof("radix_hist", s, 8.0 * n);
-    rs_hist_kernel<<<grid_for(n, T_THREADS, 4), T_THREADS, hsm, s>>>(keys, n, begin_bit, passes,
-                                                                     hist.get());
+    rs_hist_kernel<Src><<<grid_for(n, T_THREADS, 4), T_THREADS, hsm, s>>>(first, n, begin_bit, passes, hist.get());
     TC_LAUNCH_CHECK();
   }
   rs_hist_scan_kernel<<<1, 256, 0, s>>>(hist.get(), passes);
   TC_LAUNCH_CHECK();
   DevBuf<uint64_t> scratch;  // [tile counter][status ntiles*256]
   scratch.alloc(1 + ntiles * 256, s);
-  uint64_t *src = keys, *dst = tmp;
+  uint64_t *prev = nullptr;
   for (int p = 0; p < passes; ++p) {
+    uint64_t *dst = (p % 2 == 0) ? out0 : out1;
     TC_CUDA(cudaMemsetAsync(scratch.get(), 0, scratch.bytes(), s));
     ProfScope prof("radix_pass", s, 16.0 * n);
-    rs_pass_kernel<<<(unsigned)ntiles, T_THREADS, 0, s>>>(src, dst, n, begin_bit + 8 * p,
-                                                          hist.get() + p * 256, scratch.get() + 1,
-                                                          (uint32_t *)scratch.get());
+    if (p == 0) {
+      rs_pass_kernel<Src><<<(unsigned)ntiles, T_THREADS, 0, s>>>(first, dst, n, begin_bit, hist.get(),
+                                                                 scratch.get() + 1, (uint32_t *)scratch.get());
+    } else {
+      rs_pass_kernel<KeySrc><<<(unsigned)ntiles, T_THREADS, 0, s>>>(KeySrc{prev}, dst, n, begin_bit + 8 * p,
+                                                                    hist.get() + p * 256, scratch.get() + 1,
+                                                                    (uint32_t *)scratch.get());
+    }
     TC_LAUNCH_CHECK();
-    std::swap(src, dst);
+    prev = dst;
   }
-  return src;
+  return prev;
+}
+
+uint64_t *radix_sort_u64(uint64_t *keys, uint64_t *tmp, uint64_t n, int begin_bit, int end_bit, cudaStream_t s) {
+  if (n <= 1 || end_bit <= begin_bit) return keys;
+  return radix_sort_impl(KeySrc{keys}, tmp, keys, n, begin_bit, end_bit, s);
+}
+
+uint64_t *radix_sort_edges(const uint32_t *src, const uint32_t *dst, uint64_t M, uint32_t nv, int bits,
+                           uint64_t sentinel, uint64_t *buf0, uint64_t *buf1, unsigned *err, cudaStream_t s) {
+  if (M == 0) return buf0;
+  return radix_sort_impl(EdgeSrc{src, dst, nv, bits, sentinel, err}, buf0, buf1, M, 0, 2 * bits, s);
 }
 
 }  // namespace tc

@@ -14,10 +14,16 @@ void scan_u64(const uint64_t *in, uint64_t *out, uint64_t n, cudaStream_t s);
 uint64_t *radix_sort_u64(uint64_t *keys, uint64_t *tmp, uint64_t N, int begin_bit, int end_bit,
                          cudaStream_t s);
 
+// Sort of raw edge samples canonicalised on the fly (a1+a2): key (min << bits) | max,
+// self-loops / ids >= nv -> `sentinel` (ids >= nv also set *err).  Result in buf0 or buf1.
+uint64_t *radix_sort_edges(const uint32_t *src, const uint32_t *dst, uint64_t M, uint32_t nv, int bits,
+                           uint64_t sentinel, uint64_t *buf0, uint64_t *buf1, unsigned *err, cudaStream_t s);
+
 // Unique on a sorted array: out receives the first key of every run; *d_count (device)
-// receives the number of runs.
-void unique_sorted_u64(const uint64_t *in, uint64_t *out, uint64_t N, uint64_t *d_count,
-                       cudaStream_t s);
+// receives the number of runs.  deg != nullptr: also accumulate undirected degrees of the
+// kept (u << bits) | v keys other than `sentinel`.
+void unique_sorted_u64(const uint64_t *in, uint64_t *out, uint64_t N, uint64_t *d_count, cudaStream_t s,
+                       uint32_t *deg = nullptr, int bits = 0, uint64_t sentinel = 0);
 
 // Block-wide exclusive scan helper (256 threads) used by several kernels.
 template <typename T>

@@ -6,8 +6,8 @@
 //   PAPER   A-order (Algorithm 2) on the host (aorder.cpp), perm and bucket offsets uploaded
 // Oriented CSR: each undirected edge {u,v} becomes (π(src), π(dst)) with src the earlier
 // endpoint in the directing order; keys (π(src) << b) | π(dst) are radix-sorted,
-// giving ascending lists N+(x) (the layout binary search needs); offsets are the
-// exclusive scan of d~ in the new labels.
+// giving ascending lists N+(x) (the layout binary search needs); offsets come
+// from the run boundaries of π(s) in the same pass that extracts the column array.
 #include <vector>
 
 #include "internal.h"
@@ -43,21 +43,34 @@ __global__ void orient_keys_kernel(const uint64_t *__restrict__ edges, uint64_t 
   }
 }
 
-__global__ void scatter_od_kernel(const uint32_t *__restrict__ od, const uint32_t *__restrict__ perm, uint32_t n,
-                                  uint32_t *__restrict__ od_new) {
-  for (uint64_t v = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (uint64_t)gridDim.x * blockDim.x)
-    od_new[perm[v]] = od[v];
+// col[i] = low bits of the sorted (π(s) << b) | π(t) keys; offs from the run boundaries of
+// π(s) (every label in a gap gets the boundary index) — no out-degree pass needed.
+__global__ void extract_csr_kernel(const uint64_t *__restrict__ keys, uint64_t m, int bits, uint32_t n,
+                                   uint32_t *__restrict__ col, uint64_t *__restrict__ offs) {
+  const uint64_t mask = (1ull << bits) - 1;
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < m; i += (uint64_t)gridDim.x * blockDim.x) {
+    const uint64_t k = keys[i];
+    col[i] = (uint32_t)(k & mask);
+    const uint64_t s = k >> bits;
+    const uint64_t sp = i ? (keys[i - 1] >> bits) : 0;
+    if (i > 0 && s != sp)
+      for (uint64_t x = sp + 1; x <= s; ++x) offs[x] = i;  // interior gaps are short
+  }
 }
 
-__global__ void extract_col_kernel(const uint64_t *__restrict__ keys, uint64_t m, uint64_t mask,
-                                   uint32_t *__restrict__ col) {
-  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < m; i += (uint64_t)gridDim.x * blockDim.x)
-    col[i] = (uint32_t)(keys[i] & mask);
+// Labels before the first source get 0, after the last source m (long tails, e.g. the
+// d~ = 0 vertices that D-order / A-order put last, are filled grid-wide).
+__global__ void csr_ends_kernel(const uint64_t *__restrict__ keys, uint64_t m, int bits, uint32_t n,
+                                uint64_t *__restrict__ offs) {
+  const uint64_t s_first = keys[0] >> bits, s_last = keys[m - 1] >> bits;
+  for (uint64_t x = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; x <= n; x += (uint64_t)gridDim.x * blockDim.x) {
+    if (x <= s_first) offs[x] = 0;
+    else if (x > s_last) offs[x] = m;
+  }
 }
 
 }  // namespace
 
-uint32_t device_max_u32(const uint32_t *a, uint64_t n, cudaStream_t s);
 
 void build_oriented_csr(Graph &g) {
   cudaStream_t s = g.stream;
@@ -89,23 +102,17 @@ void build_oriented_csr(Graph &g) {
     tmp.alloc(m ? m : 1, s);
     sorted = radix_sort_u64(keys.get(), tmp.get(), m, 0, 2 * b, s);
   }
-  // offsets from d~ in the new labels
   g.offs.alloc((uint64_t)n + 1, s);
-  if (ident) {
-    scan_u32_to_u64(g.od.get(), g.offs.get(), n, s);
-  } else {
-    DevBuf<uint32_t> odn;
-    odn.alloc(n ? n : 1, s);
-    if (n) scatter_od_kernel<<<grid_for(n, 256), 256, 0, s>>>(g.od.get(), g.perm.get(), n, odn.get());
-    TC_LAUNCH_CHECK();
-    scan_u32_to_u64(odn.get(), g.offs.get(), n, s);
-  }
-  g.col.alloc(m + 32, s);  // tail padding: vectorised loads may over-read by < 16 B
+  g.col.alloc(m + 32, s);  // tail padding: TMA bulk copies may over-read by < 16 B
   TC_CUDA(cudaMemsetAsync(g.col.get() + m, 0xff, 32 * sizeof(uint32_t), s));
   if (m) {
-    ProfScope prof("extract_col", s, 12.0 * m);
-    extract_col_kernel<<<grid_for(m, 256), 256, 0, s>>>(sorted, m, (1ull << b) - 1, g.col.get());
+    ProfScope prof("extract_csr", s, 12.0 * m);
+    extract_csr_kernel<<<grid_for(m, 256), 256, 0, s>>>(sorted, m, b, n, g.col.get(), g.offs.get());
     TC_LAUNCH_CHECK();
+    csr_ends_kernel<<<grid_for((uint64_t)n + 1, 256), 256, 0, s>>>(sorted, m, b, n, g.offs.get());
+    TC_LAUNCH_CHECK();
+  } else {
+    TC_CUDA(cudaMemsetAsync(g.offs.get(), 0, g.offs.bytes(), s));
   }
   g.csr_ready = true;
 }
@@ -113,6 +120,7 @@ void build_oriented_csr(Graph &g) {
 void reorder_graph(Graph &g, int rule, const tc_aorder_params &p) {
   cudaStream_t s = g.stream;
   const uint32_t n = g.n;
+  if (rule != TC_REORDER_NONE) ensure_od(g);  // D-order / A-order read d~
   g.perm.release();
   g.bucket_off.release();
   g.h_bucket_off.clear();

@@ -1,0 +1,139 @@
+"""Full-size BASELINE.json configs on the GPU, in the launch configuration bench.py times.
+
+* configs[1] (ER, 67M edges): whole oracle vs GPU — oriented CSR bit-exact and T.
+* configs[2] (R-MAT s22): A-direction orientation bit-exact vs the sequential oracle
+  (sub, dsnap, CSR); T equal over ID/degree/A-direction; oracle counts on sampled vertex
+  ranges; per-vertex t(v) on sampled vertices vs the oracle's definition straight from
+  the raw samples; Σt = 3T; GPU partition bounds vs the restated work rule.
+* configs[3] (R-MAT s24 ef32): T equal over none/D-order/A-order; sampled t(v); Σt = 3T.
+* configs[4] (Kronecker s27, 2^31 samples): marked slow; same properties.
+"""
+import functools
+
+import numpy as np
+import pytest
+
+import graphgen
+import oracle
+import paper_conf_sigmod_hu0l21_b200 as tc
+from tests.test_dist_gloo import work_bounds
+
+pytestmark = pytest.mark.gpu
+
+
+@functools.lru_cache(maxsize=2)
+def samples(cfg):
+    return graphgen.generate_cpu(graphgen.CONFIGS[cfg])
+
+
+def check_local(src, dst, t_gpu, n, seed, k=400):
+    """t(v) of uniformly sampled vertex ids (chosen without looking at the GPU output)
+    against the oracle's definition from the raw samples; hubs above 2000 skipped."""
+    rng = np.random.default_rng(seed)
+    vs = np.sort(rng.choice(n, size=k, replace=False)).astype(np.uint32)
+    loc = oracle.local_triangles(src, dst, vs, max_deg=2000)
+    ok = loc != np.iinfo(np.uint64).max
+    assert ok.sum() > k // 2
+    assert np.array_equal(loc[ok], t_gpu[vs[ok]].astype(np.uint64))
+    assert (loc[ok] > 0).sum() > 0
+
+
+def test_config2_er_full_oracle():
+    spec = graphgen.CONFIGS[2]
+    src, dst = samples(2)
+    ref = oracle.run(src, dst, spec.n, "degree", "none")
+    g = tc.Graph(src, dst, spec.n).direct("degree").reorder("none")
+    offs, col, perm = g.export()
+    assert np.array_equal(offs, ref["offs"]) and np.array_equal(col, ref["col"])
+    assert g.count() == ref["T"]
+    g.free()
+
+
+def test_config3_rmat_s22():
+    spec = graphgen.CONFIGS[3]
+    n = spec.n
+    src, dst = samples(3)
+    # oracle: simple graph + sequential Alg.1 + oriented CSR (no full count: too slow on 1 core)
+    edges = oracle.simple_graph(src, dst, n)
+    dirs, info = oracle.direct(edges, n, "paper")
+    od = oracle.outdeg(edges, n, dirs)
+    perm, _ = oracle.reorder(od, "none")
+    offs, col = oracle.oriented_csr(edges, n, dirs, perm)
+    g = tc.Graph(src, dst, n).direct("paper")
+    god, sub, dsnap = g.export_direct(internals=True)
+    assert np.array_equal(sub, info["sub"]) and np.array_equal(dsnap, info["dsnap"])
+    assert np.array_equal(god, od)
+    g.reorder("none")
+    goffs, gcol, _ = g.export()
+    assert np.array_equal(goffs, offs) and np.array_equal(gcol, col)
+    T, t = g.count(per_vertex=True)
+    assert int(t.sum()) == 3 * T
+    # sampled vertex ranges of the (bit-identical) CSR counted by the oracle's merge
+    rng = np.random.default_rng(3)
+    for a in rng.integers(0, n - 40000, 3):
+        a = int(a)
+        assert g.count_range(a, a + 40000) == oracle.count_forward(offs, col, a, a + 40000)
+    check_local(src, dst, t, n, 33)
+    # work-balanced partition = the restated rule (tests/test_dist_gloo.py)
+    for world in (2, 4, 8):
+        assert g.partition(world).tolist() == work_bounds_fast(offs, col, world)
+    g.free()
+    # T does not depend on the directing rule
+    for d in ("id", "degree"):
+        g = tc.Graph(src, dst, n).direct(d).reorder("none")
+        assert g.count() == T
+        g.free()
+
+
+def work_bounds_fast(offs, col, world):
+    od = np.diff(offs.astype(np.int64))
+    s = np.zeros(len(od), np.int64)
+    nz = od > 0
+    s[nz] = np.add.reduceat(od[col.astype(np.int64)], offs[:-1][nz].astype(np.int64))
+    pre = np.concatenate([[0], np.cumsum(od + s)])
+    n = len(od)
+    b = [0] + [int(np.searchsorted(pre, (int(pre[-1]) * g) // world, side="left")) for g in range(1, world)] + [n]
+    return b
+
+
+def test_work_bounds_fast_matches_rule():
+    spec = graphgen.rmat_spec(11, 16, 3)
+    src, dst = graphgen.generate_cpu(spec)
+    res = oracle.run(src, dst, spec.n, "degree", "none")
+    for w in (2, 3, 8):
+        assert work_bounds_fast(res["offs"], res["col"], w) == work_bounds(res["offs"], res["col"], w)
+
+
+def _rules_agree(cfg, d, seed):
+    spec = graphgen.CONFIGS[cfg]
+    src, dst = samples(cfg)
+    Ts = []
+    t_ref = None
+    for r in ("none", "degree", "paper"):
+        g = tc.Graph(src, dst, spec.n).direct(d).reorder(r)
+        T, t = g.count(per_vertex=True)
+        if r == "paper":
+            b = g.export_buckets()
+            assert np.all(np.diff(b.astype(np.int64)) <= 32)
+        Ts.append(T)
+        assert int(t.sum()) == 3 * T
+        if t_ref is None:
+            t_ref = t
+        else:
+            assert np.array_equal(t, t_ref)  # per original id: reordering only relabels
+        g.free()
+    assert len(set(Ts)) == 1
+    check_local(src, dst, t_ref, spec.n, seed)
+
+
+def test_config4_rmat_s24_ef32():
+    _rules_agree(4, "degree", 44)
+
+
+@pytest.mark.slow
+def test_config5_kron_s27():
+    import os
+    mem = os.sysconf("SC_PAGE_SIZE") * os.sysconf("SC_PHYS_PAGES")
+    if mem < 96 << 30:
+        pytest.skip("host RAM too small for 2^31 CPU-generated samples")
+    _rules_agree(5, "paper", 55)

@@ -85,3 +85,21 @@ def test_count_range_partition_sums():
     cuts = [0, 100, 101, 500, 1000, spec.n]
     parts = [oracle.count_forward(res["offs"], res["col"], a, b) for a, b in zip(cuts, cuts[1:])]
     assert sum(parts) == res["T"]
+
+
+def test_local_triangles_matches_per_vertex():
+    """The sampled-vertex definition t(v) = #edges among N(v) agrees with the count's
+    per-vertex output (and brute force) on R-MAT with duplicates and self-loops."""
+    import graphgen
+    spec = graphgen.rmat_spec(12, 16, 9)
+    src, dst = graphgen.generate_cpu(spec)
+    res = oracle.run(src, dst, spec.n, "degree", "none", per_vertex=True)
+    rng = np.random.default_rng(0)
+    vs = rng.choice(spec.n, 300, replace=False).astype(np.uint32)
+    loc = oracle.local_triangles(src, dst, vs)
+    assert np.array_equal(loc, res["t"][vs])
+    rng = np.random.default_rng(1)
+    n = 50
+    s2, d2 = graphs.random_graph(rng, n, 300, "skew")
+    _, tv = graphs.brute_force(s2, d2, n)
+    assert np.array_equal(oracle.local_triangles(s2, d2, np.arange(n)).astype(np.int64), tv)
