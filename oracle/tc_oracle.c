@@ -64,19 +64,6 @@ static uint64_t edge_key(uint32_t u, uint32_t v) {
   return ((uint64_t)lo << 32) | hi;
 }
 
-/* Index of undirected edge {u,v} in the sorted edge array, or -1. */
-static int64_t edge_index(const uint64_t *edges, uint64_t m, uint32_t u, uint32_t v) {
-  uint64_t key = edge_key(u, v);
-  uint64_t lo = 0, hi = m;
-  while (lo < hi) {
-    uint64_t mid = lo + (hi - lo) / 2;
-    if (edges[mid] < key) lo = mid + 1;
-    else hi = mid;
-  }
-  if (lo < m && edges[lo] == key) return (int64_t)lo;
-  return -1;
-}
-
 /* ------------------------------------------------------------------------ */
 /* O1: simple undirected graph ("undirected graph G=(V,E)")     */
 /* ------------------------------------------------------------------------ */
@@ -176,6 +163,22 @@ int orc_direct_paper(const uint64_t *edges, uint64_t m, uint32_t n, const uint64
   uint32_t *frontier = (uint32_t *)malloc(sizeof(uint32_t) * nn);
   uint32_t *next = (uint32_t *)malloc(sizeof(uint32_t) * nn);
   for (uint32_t v = 0; v < n; ++v) d[v] = (uint32_t)(offs[v + 1] - offs[v]);
+  /* N(v) in edge order, each entry with the index of its undirected edge, so that the
+   * "(v,nbr) is unset" test is a direct lookup (the list order does not matter: frontier
+   * members are processed as a set, see readings Q7/Q9). */
+  (void)adj;
+  uint64_t *cur = (uint64_t *)malloc(sizeof(uint64_t) * nn);
+  uint32_t *nb = (uint32_t *)malloc(sizeof(uint32_t) * (2 * m + 1));
+  uint64_t *eid = (uint64_t *)malloc(sizeof(uint64_t) * (2 * m + 1));
+  for (uint32_t v = 0; v < n; ++v) cur[v] = offs[v];
+  for (uint64_t i = 0; i < m; ++i) {
+    uint32_t u = (uint32_t)(edges[i] >> 32), w = (uint32_t)edges[i];
+    nb[cur[u]] = w;
+    eid[cur[u]++] = i;
+    nb[cur[w]] = u;
+    eid[cur[w]++] = i;
+  }
+  free(cur);
 
   uint64_t npeeled = 0;
   uint32_t level = 0, subround = 0;
@@ -197,8 +200,8 @@ int orc_direct_paper(const uint64_t *edges, uint64_t m, uint32_t n, const uint64
       for (uint64_t i = 0; i < nf; ++i) {                 /* line 8 */
         uint32_t v = frontier[i];
         for (uint64_t p = offs[v]; p < offs[v + 1]; ++p) {
-          uint32_t nbr = adj[p];
-          int64_t e = edge_index(edges, m, v, nbr);
+          uint32_t nbr = nb[p];
+          uint64_t e = eid[p];
           if (isset[e]) continue;
           if (in_frontier[nbr]) {                         /* line 9 */
             int v_first = dsnap[v] < dsnap[nbr] || (dsnap[v] == dsnap[nbr] && v < nbr);
@@ -231,7 +234,7 @@ int orc_direct_paper(const uint64_t *edges, uint64_t m, uint32_t n, const uint64
   if (levels_out) *levels_out = level;
   if (subrounds_out) *subrounds_out = subround;
   free(d); free(dsnap); free(peeled); free(in_frontier); free(queued); free(isset);
-  free(frontier); free(next);
+  free(frontier); free(next); free(nb); free(eid);
   return 0;
 }
 

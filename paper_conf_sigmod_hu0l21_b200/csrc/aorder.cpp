@@ -109,6 +109,83 @@ struct PackedTournament4 {
     return t == UINT64_MAX ? -1 : (int64_t)(t & ((1ull << ib) - 1));
   }
 };
+
+// Monotone bucketed priority queue on the same packed keys.  In both phases only the
+// top bucket changes and its packed key only grows (phase 1 adds S > 0 to the min; phase
+// 2 adds S <= 0 to the max, i.e. its negated key grows), so the extracted minimum never
+// decreases: keys are binned by their high bits, only the lowest non-empty bin is kept as
+// an exact binary min-heap (small, cache-resident), higher bins are plain vectors.
+struct MonoQueue {
+  int shift = 0;
+  uint64_t bin0 = 0;
+  std::vector<std::vector<uint64_t>> bins;
+  std::vector<uint64_t> heap;
+  size_t cur = 0;
+  size_t bin_of(uint64_t pk) const { return (size_t)((pk >> shift) - bin0); }
+  void sift_down(size_t i) {
+    const size_t n = heap.size();
+    uint64_t x = heap[i];
+    for (;;) {
+      size_t c = 2 * i + 1;
+      if (c >= n) break;
+      if (c + 1 < n && heap[c + 1] < heap[c]) ++c;
+      if (heap[c] >= x) break;
+      heap[i] = heap[c];
+      i = c;
+    }
+    heap[i] = x;
+  }
+  void sift_up(size_t i) {
+    uint64_t x = heap[i];
+    while (i > 0) {
+      size_t p = (i - 1) / 2;
+      if (heap[p] <= x) break;
+      heap[i] = heap[p];
+      i = p;
+    }
+    heap[i] = x;
+  }
+  void refill() {
+    while (heap.empty() && cur + 1 < bins.size()) {
+      ++cur;
+      heap.swap(bins[cur]);
+      for (size_t i = heap.size() / 2; i-- > 0;) sift_down(i);
+    }
+  }
+  // keys: packed keys of the alive buckets; max_pk: upper bound of any key ever inserted;
+  // step: smallest key increment (packed units).  Bins ~step/8 wide so that the buckets
+  // bunched at the "water level" of phase 2 spread over many small heaps (<= 2^16 bins).
+  void build(const std::vector<uint64_t> &keys, uint64_t max_pk, uint64_t step) {
+    uint64_t mn = UINT64_MAX;
+    for (uint64_t k : keys) mn = std::min(mn, k);
+    if (keys.empty()) mn = 0;
+    const int span_bits = 64 - __builtin_clzll((max_pk - mn) | 1);
+    const int step_bits = step >= 8 ? 63 - __builtin_clzll(step / 8) : 0;
+    shift = std::max(step_bits, std::max(0, span_bits - 16));
+    bin0 = mn >> shift;
+    bins.assign(((max_pk >> shift) - bin0) + 2, {});
+    for (uint64_t k : keys) bins[bin_of(k)].push_back(k);
+    cur = 0;
+    heap.swap(bins[0]);
+    for (size_t i = heap.size() / 2; i-- > 0;) sift_down(i);
+    refill();
+  }
+  bool empty() const { return heap.empty(); }
+  uint64_t top() const { return heap[0]; }
+  // the top's key grew to `pk` (alive) or its bucket left the queue (!alive)
+  void replace_top(uint64_t pk, bool alive) {
+    if (alive && bin_of(pk) == cur) {
+      heap[0] = pk;
+      sift_down(0);
+      return;
+    }
+    heap[0] = heap.back();
+    heap.pop_back();
+    if (!heap.empty()) sift_down(0);
+    if (alive) bins[bin_of(pk)].push_back(pk);
+    refill();
+  }
+};
 }  // namespace
 
 void aorder_host(const std::vector<uint32_t> &od, const tc_aorder_params &p, std::vector<uint32_t> &perm,
@@ -147,13 +224,21 @@ void aorder_host(const std::vector<uint32_t> &od, const tc_aorder_params &p, std
   const size_t b = (nact + k - 1) / k;
   std::vector<int64_t> mem_sup(b, 0);        // line 1
   std::vector<uint32_t> fill(b, 0);
-  std::vector<uint32_t> members(b * (size_t)k);
+  std::vector<uint32_t> bucket_of(n);  // insertion record, written in iteration order
   std::vector<uint8_t> alive(b, 1);
   // Phase 1 / phase 2 priority queues.  Packed 4-ary tree when max|mem_sup| and the bucket
   // index fit 63 bits (always for the default parameters), else the generic tree.
-  int64_t smax = 0;
-  for (uint32_t v : vmem) smax = std::max<int64_t>(smax, std::llabs(S(od[v])));
-  for (uint32_t v : vcomp) smax = std::max<int64_t>(smax, std::llabs(S(od[v])));
+  int64_t smax = 0, smin1 = INT64_MAX, smin2 = INT64_MAX;  // max |S|; min nonzero |S| per phase
+  for (uint32_t v : vmem) {
+    int64_t a = std::llabs(S(od[v]));
+    smax = std::max(smax, a);
+    if (a) smin1 = std::min(smin1, a);
+  }
+  for (uint32_t v : vcomp) {
+    int64_t a = std::llabs(S(od[v]));
+    smax = std::max(smax, a);
+    if (a) smin2 = std::min(smin2, a);
+  }
   const int ib = b > 1 ? 64 - __builtin_clzll((unsigned long long)(b - 1)) : 1;
   const long double bound = (long double)smax * (long double)k * 2.0L + 2.0L;  // |mem_sup| < k smax
   const bool packed = bound * (long double)(1ull << ib) < 9.0e18L;
@@ -162,7 +247,8 @@ void aorder_host(const std::vector<uint32_t> &od, const tc_aorder_params &p, std
     q.build(b, mem_sup, alive);
     for (uint32_t v : vmem) {                // line 5
       int64_t bk = q.top();                  // line 6
-      members[(size_t)bk * k + fill[bk]++] = v;  // line 7
+      bucket_of[v] = (uint32_t)bk;          // line 7
+      fill[bk]++;
       mem_sup[bk] += S(od[v]);               // line 8
       if (fill[bk] == k) alive[bk] = 0;
       q.update((size_t)bk, mem_sup[bk], alive[bk]);  // line 9
@@ -171,7 +257,8 @@ void aorder_host(const std::vector<uint32_t> &od, const tc_aorder_params &p, std
     q.build(b, mem_sup, alive);
     for (uint32_t v : vcomp) {               // line 11
       int64_t bk = q.top();                  // line 12
-      members[(size_t)bk * k + fill[bk]++] = v;  // line 13
+      bucket_of[v] = (uint32_t)bk;          // line 13
+      fill[bk]++;
       mem_sup[bk] += S(od[v]);               // line 14
       if (fill[bk] == k) alive[bk] = 0;
       q.update((size_t)bk, mem_sup[bk], alive[bk]);  // line 15
@@ -179,25 +266,57 @@ void aorder_host(const std::vector<uint32_t> &od, const tc_aorder_params &p, std
   };
   if (b) {
     if (packed) {
-      PackedTournament4 q;
-      q.ib = ib;
-      q.off = (int64_t)(smax * (int64_t)k + 1);
-      run(q);
+      const int64_t off = (int64_t)(smax * (int64_t)k + 1);
+      const uint64_t imask = (1ull << ib) - 1;
+      const uint64_t max_pk = ((uint64_t)(2 * off) << ib) | imask;
+      auto pack = [&](size_t i, int64_t sup, bool want_max) {
+        return ((uint64_t)((want_max ? -sup : sup) + off) << ib) | (uint64_t)i;
+      };
+      MonoQueue q;
+      std::vector<uint64_t> keys;
+      keys.reserve(b);
+      for (size_t i = 0; i < b; ++i) keys.push_back(pack(i, 0, false));
+      q.build(keys, max_pk, smin1 == INT64_MAX ? 0 : (uint64_t)smin1 << ib);  // line 2: min queue
+      for (uint32_t v : vmem) {              // line 5
+        const size_t bk = (size_t)(q.top() & imask);  // line 6
+        bucket_of[v] = (uint32_t)bk;        // line 7
+        fill[bk]++;
+        mem_sup[bk] += S(od[v]);             // line 8
+        if (fill[bk] == k) alive[bk] = 0;
+        q.replace_top(pack(bk, mem_sup[bk], false), alive[bk]);  // line 9
+      }
+      keys.clear();
+      for (size_t i = 0; i < b; ++i)
+        if (alive[i]) keys.push_back(pack(i, mem_sup[i], true));
+      q.build(keys, max_pk, smin2 == INT64_MAX ? 0 : (uint64_t)smin2 << ib);  // line 10: max queue
+      for (uint32_t v : vcomp) {             // line 11
+        const size_t bk = (size_t)(q.top() & imask);  // line 12
+        bucket_of[v] = (uint32_t)bk;        // line 13
+        fill[bk]++;
+        mem_sup[bk] += S(od[v]);             // line 14
+        if (fill[bk] == k) alive[bk] = 0;
+        q.replace_top(pack(bk, mem_sup[bk], true), alive[bk]);  // line 15
+      }
     } else {
       Tournament q;
       run(q);
     }
   }
+  // line 16-20: buckets in index order, members in insertion order (a stable counting
+  // sort of the insertion record: phase-1 vertices first, each phase in iteration order)
   perm.assign(n, 0);
   bucket_off.assign(b + 1, 0);
-  uint32_t idx = 0;                          // line 16
   eq3 = 0;
-  for (size_t i = 0; i < b; ++i) {           // line 17
-    bucket_off[i] = idx;
-    for (uint32_t j = 0; j < fill[i]; ++j) perm[members[i * (size_t)k + j]] = idx++;  // line 18-20
+  for (size_t i = 0; i < b; ++i) {
+    bucket_off[i + 1] = bucket_off[i] + fill[i];
     eq3 += std::llabs(mem_sup[i]);           // Eq.3 objective (λ folded into S)
   }
-  bucket_off[b] = idx;
+  {
+    std::vector<uint32_t> cursor(bucket_off.begin(), bucket_off.end() - 1);
+    for (uint32_t v : vmem) perm[v] = cursor[bucket_of[v]]++;
+    for (uint32_t v : vcomp) perm[v] = cursor[bucket_of[v]]++;
+  }
+  uint32_t idx = bucket_off[b];
   for (size_t v = 0; v < n; ++v)
     if (od[v] == 0) perm[v] = idx++;         // Q16
 }

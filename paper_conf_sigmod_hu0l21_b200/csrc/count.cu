@@ -28,6 +28,7 @@
 namespace tc {
 
 int g_opt_small_cap = 1024;  // power of two
+int g_opt_l2_persist = 1;    // L2 access-policy window over [offs | col] during counts
 
 namespace {
 
@@ -524,6 +525,46 @@ static void configure_kernels() {
   done = true;
 }
 
+// L2 access-policy window over the head of the CSR allocation [offs | col...] for the
+// duration of the count: the offsets (8 B read per visited list, random) and as much of
+// the column array as the persisting carve-out allows stay in the 126 MB L2.  Best effort:
+// any failure just leaves the default policy.  Restored (and persisting lines released)
+// afterwards so later work on the stream is unaffected.
+struct L2Window {
+  cudaStream_t s;
+  bool on = false;
+  L2Window(cudaStream_t st, void *base, size_t bytes) : s(st) {
+    if (!g_opt_l2_persist || !bytes || !base) return;
+    int dev = 0, maxp = 0, maxw = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess ||
+        cudaDeviceGetAttribute(&maxp, cudaDevAttrMaxPersistingL2CacheSize, dev) != cudaSuccess ||
+        cudaDeviceGetAttribute(&maxw, cudaDevAttrMaxAccessPolicyWindowSize, dev) != cudaSuccess || maxp <= 0 ||
+        maxw <= 0) {
+      cudaGetLastError();
+      return;
+    }
+    size_t cur = 0;
+    if (cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize) == cudaSuccess && cur < (size_t)maxp)
+      cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, (size_t)maxp);
+    cudaStreamAttrValue v = {};
+    v.accessPolicyWindow.base_ptr = base;
+    v.accessPolicyWindow.num_bytes = std::min(bytes, std::min((size_t)maxp, (size_t)maxw));
+    v.accessPolicyWindow.hitRatio = 1.0f;
+    v.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+    v.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+    on = cudaStreamSetAttribute(s, cudaStreamAttributeAccessPolicyWindow, &v) == cudaSuccess;
+    cudaGetLastError();
+  }
+  ~L2Window() {
+    if (!on) return;
+    cudaStreamAttrValue v = {};
+    v.accessPolicyWindow.num_bytes = 0;
+    cudaStreamSetAttribute(s, cudaStreamAttributeAccessPolicyWindow, &v);
+    cudaCtxResetPersistingL2Cache();
+    cudaGetLastError();
+  }
+};
+
 static int occupancy(const void *fn, int threads, size_t smem) {
   int blocks = 0;
   TC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&blocks, fn, threads, smem));
@@ -547,6 +588,7 @@ uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *
     TC_CUDA(cudaEventCreate(&e0));
     TC_CUDA(cudaEventCreate(&e1));
   }
+  L2Window l2win(s, g.csr_mem.get(), g.csr_mem.bytes());
   if (ub < ue && g.m) {
     if (sched == TC_SCHED_RANGE) {
       const uint32_t *boff = nullptr;

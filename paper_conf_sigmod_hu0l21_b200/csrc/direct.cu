@@ -256,6 +256,7 @@ void direct_graph(Graph &g, int rule) {
   g.eq3 = -1;
   g.offs.release();
   g.col.release();
+  g.csr_mem.release();
   g.csr_ready = false;
   g.state = G_DIRECTED;
 }

@@ -13,6 +13,15 @@ enum GraphState { G_BUILT = 0, G_DIRECTED = 1, G_ORDERED = 2 };
 
 struct StageTimer;  // CUDA-event stage timing (api.cu)
 
+template <typename T>
+struct View {  // non-owning slice of a DevBuf
+  T *p = nullptr;
+  size_t n = 0;
+  T *get() const { return p; }
+  size_t bytes() const { return n * sizeof(T); }
+  void release() { p = nullptr; n = 0; }
+};
+
 struct Graph {
   int device = 0;
   cudaStream_t stream = nullptr;
@@ -43,8 +52,11 @@ struct Graph {
   std::vector<uint32_t> h_bucket_off;  // A-order buckets (host)
   DevBuf<uint32_t> bucket_off;    // A-order buckets (device)
   int64_t eq3 = -1;
-  DevBuf<uint64_t> offs;          // n+1
-  DevBuf<uint32_t> col;           // m (+ 8 padding words)
+  // oriented CSR in ONE allocation [offs (n+1) u64 | col (m+32) u32] so that one L2
+  // access-policy window can keep the offsets (random, 8 B per list) resident
+  DevBuf<uint64_t> csr_mem;
+  View<uint64_t> offs;            // n+1
+  View<uint32_t> col;             // m (+ 32 padding words)
   bool csr_ready = false;
 
   // a8 schedule
@@ -79,5 +91,6 @@ void analyze_graph(Graph &g);
 // options (api.cu)
 extern int g_opt_profile;
 extern int g_opt_small_cap;
+extern int g_opt_l2_persist;
 
 }  // namespace tc

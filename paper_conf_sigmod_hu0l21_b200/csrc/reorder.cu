@@ -102,8 +102,14 @@ void build_oriented_csr(Graph &g) {
     tmp.alloc(m ? m : 1, s);
     sorted = radix_sort_u64(keys.get(), tmp.get(), m, 0, 2 * b, s);
   }
-  g.offs.alloc((uint64_t)n + 1, s);
-  g.col.alloc(m + 32, s);  // tail padding: TMA bulk copies may over-read by < 16 B
+  // [offs | col] in one allocation; col gets 32 words of tail padding (TMA bulk copies may
+  // over-read by < 16 B) and starts 16-B aligned
+  const uint64_t offs_words = ((uint64_t)n + 1 + 1) & ~1ull;
+  g.offs.release();
+  g.col.release();
+  g.csr_mem.alloc(offs_words + (m + 32 + 1) / 2, s);
+  g.offs = View<uint64_t>{g.csr_mem.get(), (size_t)n + 1};
+  g.col = View<uint32_t>{reinterpret_cast<uint32_t *>(g.csr_mem.get() + offs_words), (size_t)(m + 32)};
   TC_CUDA(cudaMemsetAsync(g.col.get() + m, 0xff, 32 * sizeof(uint32_t), s));
   if (m) {
     ProfScope prof("extract_csr", s, 12.0 * m);

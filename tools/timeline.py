@@ -14,6 +14,10 @@ dst = torch.empty(spec.samples, dtype=torch.int32, device="cuda")
 graphgen.generate_cuda(spec, src.data_ptr(), dst.data_ptr(), torch.cuda.current_stream().cuda_stream)
 torch.cuda.synchronize()
 prm, keep = tc.make_aorder_params()
+import os
+for kv in filter(None, os.environ.get("TC_OPTS", "").split(",")):
+    k, v = kv.split("=")
+    tc.tc_set_option(k, int(v))
 for it in range(4):
     tc.tc_set_option("kernel_profile", 1)
     tc.tc_profile_report(reset=True)
