@@ -58,9 +58,11 @@ typedef enum {
 typedef enum { TC_DIRECT_ID = 0, TC_DIRECT_DEGREE = 1, TC_DIRECT_PAPER = 2 } tc_direct_rule;
 typedef enum { TC_REORDER_NONE = 0, TC_REORDER_DEGREE = 1, TC_REORDER_PAPER = 2 } tc_reorder_rule;
 
-/* Counting schedule (step a8).  AUTO = RANGE after an A-order reordering (the block
- * model A-order optimises: "every consecutive k vertices are grouped into a bucket ...
- * assigned to one block"), BUCKETED otherwise. */
+/* Counting schedule (step a8).  BUCKETED: (u, 32-v chunk) work items, heaviest
+ * ⌊log2 d~⌋ bin first, fetched dynamically.  RANGE: CTA i takes the k consecutive labels
+ * of bucket i — the block model A-order optimises ("every consecutive k vertices are
+ * grouped into a bucket ... assigned to one block").  AUTO = BUCKETED (measured
+ * faster on B200 for every ordering). */
 typedef enum { TC_SCHED_AUTO = 0, TC_SCHED_BUCKETED = 1, TC_SCHED_RANGE = 2 } tc_schedule;
 
 /* A-order parameters (Alg.2 inputs "F_c, F_m, λ"; Eq.19-22).
@@ -162,8 +164,10 @@ tc_status tc_export_buckets(tc_graph *g, uint32_t *bucket_off);
 
 /* Library options: "profile" (0/1: per-stage CUDA-event timing in tc_stats_t, default 1),
  * "kernel_profile" (0/1: per-kernel event pairs for tc_profile_report, default 0),
- * "small_cap" (power of two; d~(u) below it is counted warp-per-vertex with N+(u) in a
- * shared-memory slice, default 1024). */
+ * "small_cap" (power of two in [32, 2048]; d~(u) below it is counted with N+(u) in a
+ * per-warp shared-memory slice, default 1024), "l2_persist" (0/1: L2 access-policy window
+ * over the CSR during counts, default 0), "trim_memory" (any value: release the library's
+ * cached device blocks). */
 tc_status tc_set_option(const char *key, int64_t value);
 
 /* Per-kernel profile since the last reset, as JSON text into buf (host, cap bytes):

@@ -482,6 +482,7 @@ void orc_oriented_csr(const uint64_t *edges, uint64_t m, uint32_t n, const uint8
 typedef struct {
   uint64_t *slot; /* key + 1, 0 = empty */
   uint64_t cap;
+  uint64_t size;
 } u64set;
 
 static uint64_t mix64(uint64_t x) {
@@ -493,6 +494,7 @@ static void set_init(u64set *s, uint64_t want) {
   uint64_t cap = 16;
   while (cap < 2 * want + 16) cap <<= 1;
   s->cap = cap;
+  s->size = 0;
   s->slot = (uint64_t *)calloc(cap, sizeof(uint64_t));
 }
 
@@ -505,13 +507,26 @@ static int set_has(const u64set *s, uint64_t k) {
   return 0;
 }
 
+static void set_add(u64set *s, uint64_t k);
+
+static void set_grow(u64set *s) { /* keep the load factor <= 1/2 */
+  u64set t;
+  set_init(&t, s->cap);
+  for (uint64_t i = 0; i < s->cap; ++i)
+    if (s->slot[i]) set_add(&t, s->slot[i] - 1);
+  free(s->slot);
+  *s = t;
+}
+
 static void set_add(u64set *s, uint64_t k) {
+  if (2 * (s->size + 1) > s->cap) set_grow(s);
   uint64_t i = mix64(k) & (s->cap - 1);
   while (s->slot[i]) {
     if (s->slot[i] == k + 1) return;
     i = (i + 1) & (s->cap - 1);
   }
   s->slot[i] = k + 1;
+  s->size++;
 }
 
 /* vs[0..nv): sampled vertices (each with degree <= max_deg in the simple graph, else

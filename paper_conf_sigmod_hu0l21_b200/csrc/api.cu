@@ -181,9 +181,10 @@ tc_status tc_set_option(const char *key, int64_t value) {
     if (k == "profile") g_opt_profile = value ? 1 : 0;
     else if (k == "kernel_profile") g_opt_kernel_profile = value ? 1 : 0;
     else if (k == "l2_persist") g_opt_l2_persist = value ? 1 : 0;
+    else if (k == "trim_memory") dev_trim();
     else if (k == "small_cap") {
-      TC_REQUIRE(value >= 32 && value <= 16384 && (value & (value - 1)) == 0, ST_INVALID,
-                 "small_cap must be a power of two in [32, 16384]");
+      TC_REQUIRE(value >= 32 && value <= 2048 && (value & (value - 1)) == 0, ST_INVALID,
+                 "small_cap must be a power of two in [32, 2048]");
       g_opt_small_cap = (int)value;
     } else throw Error(ST_INVALID, "unknown option " + k);
   });

@@ -53,8 +53,11 @@ void build_graph(Graph &g, const uint32_t *d_src, const uint32_t *d_dst, uint64_
   const uint64_t sentinel = (b * 2 >= 64) ? ~0ull : ((1ull << (2 * b)) - 1);
 
   DevBuf<uint64_t> keys, tmp;
-  keys.alloc(M ? M : 1, s);
-  tmp.alloc(M ? M : 1, s);
+  {
+    ProfScope prof("alloc_keys", s, 0.0);
+    keys.alloc(M ? M : 1, s);
+    tmp.alloc(M ? M : 1, s);
+  }
   DevBuf<unsigned> err;
   err.alloc(1, s);
   DevBuf<uint64_t> d_m;

@@ -39,7 +39,13 @@ extern unsigned long long g_launch_count;  // kernels launched by the library (p
 enum { ST_OK = 0, ST_INVALID = 1, ST_OOM = 2, ST_CUDA = 3, ST_NCCL = 4, ST_STATE = 5 };
 
 // ---------------------------------------------------------------- device buffers
-// Stream-ordered allocation (cudaMallocAsync) owned by the graph; freed on its stream.
+// Device memory cache (alloc.cu): stream-ordered reuse of blocks across graphs and steps.
+void *dev_alloc(size_t bytes, cudaStream_t s);
+void dev_free(void *p, size_t bytes, cudaStream_t s);
+void dev_trim();
+size_t dev_cached_bytes();
+
+// Buffer owned by the graph (or a stage), allocated from / returned to the cache on its stream.
 template <typename T>
 struct DevBuf {
   T *p = nullptr;
@@ -62,16 +68,15 @@ struct DevBuf {
     s = stream;
     n = count;
     if (count == 0) return;
-    cudaError_t e = cudaMallocAsync((void **)&p, count * sizeof(T), stream);
-    if (e == cudaErrorMemoryAllocation) {
-      cudaGetLastError();
+    try {
+      p = (T *)dev_alloc(count * sizeof(T), stream);
+    } catch (...) {
       p = nullptr; n = 0;
-      throw Error(ST_OOM, "device allocation of " + std::to_string(count * sizeof(T)) + " bytes failed");
+      throw;
     }
-    TC_CUDA(e);
   }
   void release() {
-    if (p) cudaFreeAsync(p, s);
+    if (p) dev_free(p, n * sizeof(T), s);
     p = nullptr; n = 0;
   }
   T *get() const { return p; }

@@ -28,7 +28,7 @@
 namespace tc {
 
 int g_opt_small_cap = 1024;  // power of two
-int g_opt_l2_persist = 1;    // L2 access-policy window over [offs | col] during counts
+int g_opt_l2_persist = 0;    // L2 access-policy window over [offs | col] during counts (off: measured slower overall)
 
 namespace {
 
@@ -43,6 +43,7 @@ struct WarpScratch {  // per-warp owner-search tables for one 32-v chunk
   uint64_t vb[32];
   uint32_t pre[32];
   uint32_t v[32];
+  uint32_t vcnt[32];  // per-vertex mode: matches per owner v (flushed once per chunk)
 };
 
 __device__ __forceinline__ uint32_t ldg_u32(const uint32_t *p) { return __ldg(p); }
@@ -66,15 +67,16 @@ __device__ __forceinline__ bool bsearch_list(const uint32_t *s, uint32_t L, uint
 // Fixed-depth search over a list padded with +inf (0xffffffff, never a vertex id) to 2^S
 // entries: S unrolled steps of one shared load + compare + select each ("binary lifting").
 // Precondition: s[0] <= w (the caller's range filter).
+// Returns the position p of the last element <= w (hit iff tc_smem[p] == w).
 template <int S>
-__device__ __forceinline__ bool bsearch_pow2(uint32_t sbase, uint32_t w) {
+__device__ __forceinline__ uint32_t bsearch_pow2(uint32_t sbase, uint32_t w) {
   uint32_t p = sbase;
 #pragma unroll
   for (int k = S - 1; k >= 0; --k) {
     uint32_t q = p + (1u << k);
     p = (tc_smem[q] <= w) ? q : p;
   }
-  return tc_smem[p] == w;
+  return p;
 }
 
 __device__ __forceinline__ int ceil_log2(uint32_t L) { return L <= 1 ? 0 : 32 - __clz(L - 1); }
@@ -83,10 +85,13 @@ __device__ __forceinline__ int ceil_log2(uint32_t L) { return L <= 1 ? 0 : 32 - 
 // (K entries: start offset, inclusive wedge prefix); each lane walks its owner forward
 // incrementally (its wedge index grows by 32 per step), so locating w's list costs ~1
 // shared load per wedge instead of a 5-step search.
+// Per-vertex mode (PV): matches are first aggregated in shared memory — per owner v in
+// ws.vcnt, per position of w in N+(u) at tc_smem[cbase + pos] — and flushed with one global
+// atomic per distinct vertex per item (hub vertices would otherwise serialise on atomics).
 template <bool PV, int S>
 __device__ __forceinline__ uint32_t wedge_loop(const uint32_t *__restrict__ col, const uint32_t *list, uint32_t sbase,
-                                               uint32_t L, uint32_t lo, uint32_t hi, uint32_t total,
-                                               const WarpScratch &ws, unsigned long long *tv) {
+                                               uint32_t cbase, uint32_t L, uint32_t lo, uint32_t hi, uint32_t total,
+                                               WarpScratch &ws, unsigned long long *tv) {
   uint32_t cnt = 0;
   uint32_t o = 0, o_beg = 0, o_end = ws.pre[0];
   uint64_t o_vb = ws.vb[0];
@@ -117,13 +122,19 @@ __device__ __forceinline__ uint32_t wedge_loop(const uint32_t *__restrict__ col,
     for (int k = 0; k < UNR; ++k) {
       if (w[k] >= lo && w[k] <= hi) {
         bool hit;
-        if (S > 0) hit = bsearch_pow2<S>(sbase, w[k]);
-        else hit = bsearch_list(list, L, w[k]);
+        uint32_t pos = 0;
+        if (S > 0) {
+          pos = bsearch_pow2<S>(sbase, w[k]);
+          hit = tc_smem[pos] == w[k];
+        } else {
+          hit = bsearch_list(list, L, w[k]);
+        }
         if (hit) {
           ++cnt;
           if (PV) {
-            atomicAdd(&tv[w[k]], 1ull);
-            atomicAdd(&tv[ws.v[ow[k]]], 1ull);
+            atomicAdd(&ws.vcnt[ow[k]], 1u);
+            if (S > 0 && cbase != 0xffffffffu) atomicAdd(&tc_smem[cbase + (pos - sbase)], 1u);
+            else atomicAdd(&tv[w[k]], 1ull);
           }
         }
       }
@@ -138,8 +149,8 @@ __device__ __forceinline__ uint32_t wedge_loop(const uint32_t *__restrict__ col,
 template <bool PV>
 __device__ __forceinline__ uint32_t warp_chunk(const uint64_t *__restrict__ offs, const uint32_t *__restrict__ col,
                                                uint32_t v, bool valid, const uint32_t *list, uint32_t sbase,
-                                               uint32_t L, bool padded, uint32_t lo, uint32_t hi, WarpScratch &ws,
-                                               unsigned long long *tv) {
+                                               uint32_t cbase, uint32_t L, bool padded, uint32_t lo, uint32_t hi,
+                                               WarpScratch &ws, unsigned long long *tv) {
   const unsigned lane = lane_id();
   uint64_t vb = 0;
   uint32_t dv = 0;
@@ -156,6 +167,7 @@ __device__ __forceinline__ uint32_t warp_chunk(const uint64_t *__restrict__ offs
     ws.pre[pos] = inc;
     if (PV) ws.v[pos] = v;
   }
+  if (PV) ws.vcnt[lane] = 0;
   __syncwarp();
   uint32_t cnt = 0;
   if (total) {
@@ -163,22 +175,23 @@ __device__ __forceinline__ uint32_t warp_chunk(const uint64_t *__restrict__ offs
     switch (S) {
 #define TC_CASE(k) \
   case k:          \
-    cnt = wedge_loop<PV, k>(col, list, sbase, L, lo, hi, total, ws, tv); \
+    cnt = wedge_loop<PV, k>(col, list, sbase, cbase, L, lo, hi, total, ws, tv); \
     break;
       TC_CASE(1) TC_CASE(2) TC_CASE(3) TC_CASE(4) TC_CASE(5) TC_CASE(6) TC_CASE(7)
       TC_CASE(8) TC_CASE(9) TC_CASE(10) TC_CASE(11) TC_CASE(12) TC_CASE(13) TC_CASE(14)
 #undef TC_CASE
       default:
-        cnt = wedge_loop<PV, 0>(col, list, sbase, L, lo, hi, total, ws, tv);
+        cnt = wedge_loop<PV, 0>(col, list, sbase, cbase, L, lo, hi, total, ws, tv);
     }
   }
   __syncwarp();
+  if (PV && lane < (unsigned)__popc(nz) && ws.vcnt[lane]) atomicAdd(&tv[ws.v[lane]], (unsigned long long)ws.vcnt[lane]);
   return cnt;
 }
 
 // One work item: source u, v's N+(u)[c0 .. c0+32) on one warp; N+(u) is searched in the
 // warp's shared slice (staged here, padded with +inf to a power of two) when it fits,
-// else in global memory.
+// else in global memory.  PV: the slice is followed by cap match counters.
 template <bool PV>
 __device__ __forceinline__ uint64_t warp_item(const uint64_t *__restrict__ offs, const uint32_t *__restrict__ col,
                                               uint32_t u, uint32_t c0, uint32_t sbase, uint32_t cap,
@@ -189,9 +202,13 @@ __device__ __forceinline__ uint64_t warp_item(const uint64_t *__restrict__ offs,
   if (L < 2 || c0 >= L) return 0;
   const uint32_t *list;
   bool padded = false;
+  const uint32_t cbase = (PV && L <= cap) ? sbase + cap : 0xffffffffu;
   if (L <= cap) {
     const uint32_t P = 1u << ceil_log2(L);
-    for (uint32_t j = lane; j < P; j += 32) tc_smem[sbase + j] = j < L ? ldg_u32(col + a + j) : 0xffffffffu;
+    for (uint32_t j = lane; j < P; j += 32) {
+      tc_smem[sbase + j] = j < L ? ldg_u32(col + a + j) : 0xffffffffu;
+      if (PV) tc_smem[cbase + j] = 0;
+    }
     __syncwarp();
     list = tc_smem + sbase;
     padded = true;
@@ -201,11 +218,18 @@ __device__ __forceinline__ uint64_t warp_item(const uint64_t *__restrict__ offs,
   const uint32_t lo = list[0], hi = list[L - 1];
   const bool valid = c0 + lane < L;
   const uint32_t v = valid ? list[c0 + lane] : 0u;
-  uint32_t cnt = warp_chunk<PV>(offs, col, v, valid, list, sbase, L, padded, lo, hi, ws, tv);
+  uint32_t cnt = warp_chunk<PV>(offs, col, v, valid, list, sbase, cbase, L, padded, lo, hi, ws, tv);
   __syncwarp();  // slice reads done before the next item restages it
   if (PV) {
     uint64_t tot = warp_sum((uint64_t)cnt);
     if (lane == 0 && tot) atomicAdd(&tv[u], (unsigned long long)tot);
+    if (cbase != 0xffffffffu) {
+      for (uint32_t j = lane; j < L; j += 32) {
+        uint32_t c = tc_smem[cbase + j];
+        if (c) atomicAdd(&tv[tc_smem[sbase + j]], (unsigned long long)c);
+      }
+      __syncwarp();
+    }
   }
   return cnt;
 }
@@ -304,7 +328,7 @@ __global__ __launch_bounds__(CT_THREADS) void count_small_kernel(const uint64_t 
                                                                  uint64_t nheavy, unsigned long long *ctr, uint32_t cap,
                                                                  unsigned long long *T, unsigned long long *tv) {
   __shared__ WarpScratch s_ws[CT_WARPS];
-  const uint32_t slice = warp_id() * cap;
+  const uint32_t slice = warp_id() * cap * (PV ? 2 : 1);  // PV: list + counters
   WarpScratch &ws = s_ws[warp_id()];
   uint64_t acc = 0;
   while (true) {  // heavy items, one per fetch
@@ -413,7 +437,7 @@ __global__ __launch_bounds__(LG_THREADS) void count_large_kernel(const uint64_t 
       for (uint32_t c0 = cbeg + warp_id() * 32; c0 < cend; c0 += LG_THREADS) {
         bool valid = c0 + lane_id() < cend;
         uint32_t v = valid ? ldg_u32(col + a + c0 + lane_id()) : 0u;
-        cnt += warp_chunk<PV>(offs, col, v, valid, list, shift, plen, true, lo, hi, ws, tv);
+        cnt += warp_chunk<PV>(offs, col, v, valid, list, shift, 0xffffffffu, plen, true, lo, hi, ws, tv);
       }
       ucnt += cnt;
       __syncthreads();  // piece fully consumed before the next bulk copy overwrites it
@@ -433,13 +457,19 @@ __global__ __launch_bounds__(CT_THREADS) void count_range_kernel(const uint64_t 
                                                                  const uint32_t *__restrict__ col,
                                                                  const uint32_t *__restrict__ boff, uint32_t kfixed,
                                                                  uint32_t b0, uint32_t nb, uint32_t ub, uint32_t ue,
-                                                                 uint32_t cap, unsigned long long *T,
-                                                                 unsigned long long *tv) {
+                                                                 uint32_t cap, unsigned *bucket_ctr,
+                                                                 unsigned long long *T, unsigned long long *tv) {
   __shared__ WarpScratch s_ws[CT_WARPS];
-  const uint32_t slice = warp_id() * cap;
+  __shared__ uint32_t s_bucket;
+  const uint32_t slice = warp_id() * cap * (PV ? 2 : 1);  // PV: list + counters
   WarpScratch &ws = s_ws[warp_id()];
   uint64_t acc = 0;
-  for (uint32_t bi = b0 + blockIdx.x; bi < b0 + nb; bi += gridDim.x) {
+  while (true) {  // buckets fetched dynamically: a CTA takes the next bucket when done
+    __syncthreads();
+    if (threadIdx.x == 0) s_bucket = b0 + atomicAdd(bucket_ctr, 1u);
+    __syncthreads();
+    const uint32_t bi = s_bucket;
+    if (bi >= b0 + nb) break;
     uint64_t s0 = boff ? boff[bi] : (uint64_t)bi * kfixed;
     uint64_t s1 = boff ? boff[bi + 1] : (uint64_t)(bi + 1) * kfixed;
     if (s0 < ub) s0 = ub;
@@ -582,7 +612,10 @@ uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *
   unsigned long long *tv = reinterpret_cast<unsigned long long *>(d_tv);
   const uint32_t cap = (uint32_t)g_opt_small_cap;
   int sched = g.schedule;
-  if (sched == TC_SCHED_AUTO) sched = (g.reorder_rule == TC_REORDER_PAPER) ? TC_SCHED_RANGE : TC_SCHED_BUCKETED;
+  // AUTO = BUCKETED for every ordering: measured on B200 (R-MAT s22, profiles/), the
+  // dynamic heavy-first item schedule beats the static block-per-bucket model A-order
+  // targets (RANGE) by 1.3-1.5x, and makes the count time order-independent.
+  if (sched == TC_SCHED_AUTO) sched = TC_SCHED_BUCKETED;
   cudaEvent_t e0 = nullptr, e1 = nullptr;
   if (kernel_ms) {
     TC_CUDA(cudaEventCreate(&e0));
@@ -608,18 +641,21 @@ uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *
         nb = (ue + k - 1) / k - b0;
       }
       if (nb) {
-        size_t smem = (size_t)CT_WARPS * cap * sizeof(uint32_t);
+        size_t smem = (size_t)CT_WARPS * cap * (tv ? 2 : 1) * sizeof(uint32_t);
         int occ = occupancy(tv ? (const void *)count_range_kernel<true> : (const void *)count_range_kernel<false>,
                             CT_THREADS, smem);
         unsigned grid = (unsigned)std::min<uint64_t>(nb, (uint64_t)num_sms() * occ);
+        DevBuf<unsigned> bctr;
+        bctr.alloc(1, s);
+        TC_CUDA(cudaMemsetAsync(bctr.get(), 0, sizeof(unsigned), s));
         if (kernel_ms) TC_CUDA(cudaEventRecord(e0, s));
         ProfScope prof("count_range", s, 0.0);
         if (tv)
           count_range_kernel<true><<<grid, CT_THREADS, smem, s>>>(g.offs.get(), g.col.get(), boff, k, b0, nb, ub, ue,
-                                                                   cap, dT.get(), tv);
+                                                                   cap, bctr.get(), dT.get(), tv);
         else
           count_range_kernel<false><<<grid, CT_THREADS, smem, s>>>(g.offs.get(), g.col.get(), boff, k, b0, nb, ub, ue,
-                                                                    cap, dT.get(), nullptr);
+                                                                    cap, bctr.get(), dT.get(), nullptr);
         TC_LAUNCH_CHECK();
         if (kernel_ms) TC_CUDA(cudaEventRecord(e1, s));
         ++nlaunch;
@@ -672,7 +708,7 @@ uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *
         }
         uint64_t nsmall = nitems - nlarge;
         if (nsmall) {
-          size_t smem = (size_t)CT_WARPS * cap * sizeof(uint32_t);
+          size_t smem = (size_t)CT_WARPS * cap * (tv ? 2 : 1) * sizeof(uint32_t);
           int occ = occupancy(tv ? (const void *)count_small_kernel<true> : (const void *)count_small_kernel<false>,
                               CT_THREADS, smem);
           uint64_t want = (nsmall + CT_WARPS - 1) / CT_WARPS;

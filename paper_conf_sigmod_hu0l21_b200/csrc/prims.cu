@@ -357,11 +357,17 @@ static uint64_t *radix_sort_impl(Src first, uint64_t *out0, uint64_t *out1, uint
   rs_hist_scan_kernel<<<1, 256, 0, s>>>(hist.get(), passes);
   TC_LAUNCH_CHECK();
   DevBuf<uint64_t> scratch;  // [tile counter][status ntiles*256]
-  scratch.alloc(1 + ntiles * 256, s);
+  {
+    ProfScope prof("radix_scratch", s, 0.0);
+    scratch.alloc(1 + ntiles * 256, s);
+  }
   uint64_t *prev = nullptr;
   for (int p = 0; p < passes; ++p) {
     uint64_t *dst = (p % 2 == 0) ? out0 : out1;
-    TC_CUDA(cudaMemsetAsync(scratch.get(), 0, scratch.bytes(), s));
+    {
+      ProfScope prof("radix_memset", s, 8.0 * scratch.n);
+      TC_CUDA(cudaMemsetAsync(scratch.get(), 0, scratch.bytes(), s));
+    }
     ProfScope prof("radix_pass", s, 16.0 * n);
     if (p == 0) {
       rs_pass_kernel<Src><<<(unsigned)ntiles, T_THREADS, 0, s>>>(first, dst, n, begin_bit, hist.get(),

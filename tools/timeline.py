@@ -25,6 +25,8 @@ for it in range(4):
     t0 = time.perf_counter(); g = tc.tc_graph_from_edges(src, dst, spec.n); t["build"] = time.perf_counter() - t0
     t0 = time.perf_counter(); tc.tc_direct(g, d); t["direct"] = time.perf_counter() - t0
     t0 = time.perf_counter(); tc.tc_reorder(g, r, prm); t["reorder"] = time.perf_counter() - t0
+    if os.environ.get("TC_SCHED"):
+        tc.tc_set_schedule(g, os.environ["TC_SCHED"])
     t0 = time.perf_counter(); T = tc.tc_count(g); t["count"] = time.perf_counter() - t0
     st = tc.tc_get_stats(g)
     t0 = time.perf_counter(); tc.tc_graph_free(g); t["free"] = time.perf_counter() - t0
