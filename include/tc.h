@@ -165,7 +165,7 @@ tc_status tc_export_buckets(tc_graph *g, uint32_t *bucket_off);
 /* Library options: "profile" (0/1: per-stage CUDA-event timing in tc_stats_t, default 1),
  * "kernel_profile" (0/1: per-kernel event pairs for tc_profile_report, default 0),
  * "small_cap" (power of two in [32, 2048]; d~(u) below it is counted with N+(u) in a
- * per-warp shared-memory slice, default 1024), "l2_persist" (0/1: L2 access-policy window
+ * per-warp shared-memory slice, default 256), "l2_persist" (0/1: L2 access-policy window
  * over the CSR during counts, default 0), "trim_memory" (any value: release the library's
  * cached device blocks). */
 tc_status tc_set_option(const char *key, int64_t value);

@@ -133,6 +133,12 @@ __device__ __forceinline__ T warp_sum(T v) {
   return v;
 }
 
+__device__ __forceinline__ uint32_t warp_max(uint32_t v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v = max(v, __shfl_xor_sync(0xffffffffu, v, o));
+  return v;
+}
+
 template <typename T>
 __device__ __forceinline__ T warp_inclusive_scan(T v) {
   unsigned l = lane_id();

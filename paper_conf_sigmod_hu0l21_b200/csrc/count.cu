@@ -27,16 +27,18 @@
 
 namespace tc {
 
-int g_opt_small_cap = 1024;  // power of two
+int g_opt_small_cap = 256;   // power of two: d~ below it -> warp items, else CTA items
+int g_opt_bracket = 1;       // bracketed binary search for long staged lists
 int g_opt_l2_persist = 0;    // L2 access-policy window over [offs | col] during counts (off: measured slower overall)
 
 namespace {
 
 constexpr int CT_THREADS = 256;       // small / range kernels: 8 warps
 constexpr int CT_WARPS = CT_THREADS / 32;
-constexpr int LG_THREADS = 512;       // large kernel: 16 warps
+constexpr int LG_THREADS = 256;       // large kernel: 8 warps
 constexpr int LG_WARPS = LG_THREADS / 32;
-constexpr uint32_t PIECE = 16384;     // large kernel: N+(u) piece in shared memory (64 KB)
+constexpr uint32_t PIECE = 4096;      // large kernel: N+(u) piece in shared memory (16 KB)
+constexpr uint32_t LG_SMEM_WORDS = (PIECE + 72) + (PIECE + 64) / 2;  // piece (+pad) + u16 bracket table
 constexpr uint32_t CHUNK = 8;         // worklist entries per atomic fetch
 
 struct WarpScratch {  // per-warp owner-search tables for one 32-v chunk
@@ -81,6 +83,51 @@ __device__ __forceinline__ uint32_t bsearch_pow2(uint32_t sbase, uint32_t w) {
 
 __device__ __forceinline__ int ceil_log2(uint32_t L) { return L <= 1 ? 0 : 32 - __clz(L - 1); }
 
+// words of dynamic shared memory per warp in the warp-item kernels
+// (slice cap+64 words, u16 bracket table cap+64 entries, PV counters cap words)
+__host__ __device__ constexpr uint32_t warp_stride(uint32_t cap, bool pv) {
+  return (cap + 64) + (cap + 64) / 2 + (pv ? cap : 0);
+}
+
+__constant__ int g_bracket = 1;  // bracketed binary search on (option "bracket")
+
+// Searchers: does w occur in N+(u)?  `pos` = its shared-memory index (PV counters).
+struct GlobalSearch {  // N+(u) in global memory (lists longer than a warp slice)
+  const uint32_t *list;
+  uint32_t L;
+  __device__ __forceinline__ bool operator()(uint32_t w, uint32_t &pos) const {
+    pos = 0;
+    return bsearch_list(list, L, w);
+  }
+};
+template <int S>
+struct Pow2Search {  // full fixed-depth binary search over the +inf-padded slice
+  uint32_t sbase;
+  __device__ __forceinline__ bool operator()(uint32_t w, uint32_t &pos) const {
+    pos = bsearch_pow2<S>(sbase, w);
+    return tc_smem[pos] == w;
+  }
+};
+// Bracketed binary search: a per-item table maps the value bucket (w - lo) >> sh to the
+// first list position of that bucket; the binary search then only spans the bucket
+// (S2 = ceil(log2 max bucket occupancy) steps instead of ceil(log2 d~(u))).  Elements
+// past the bucket are larger than w (buckets are monotone), and the slice carries +inf
+// padding past its end, so no bounds checks are needed.
+template <int S2>
+struct TabSearch {
+  uint32_t sbase, tbase, lo, sh;
+  __device__ __forceinline__ bool operator()(uint32_t w, uint32_t &pos) const {
+    uint32_t p = sbase + reinterpret_cast<const uint16_t *>(tc_smem + tbase)[(w - lo) >> sh];
+#pragma unroll
+    for (int k = S2 - 1; k >= 0; --k) {
+      uint32_t q = p + (1u << k);
+      p = (tc_smem[q] <= w) ? q : p;
+    }
+    pos = p;
+    return tc_smem[p] == w;
+  }
+};
+
 // Wedge loop of one chunk.  Owner tables hold only the non-empty N+(v) of the chunk
 // (K entries: start offset, inclusive wedge prefix); each lane walks its owner forward
 // incrementally (its wedge index grows by 32 per step), so locating w's list costs ~1
@@ -88,9 +135,9 @@ __device__ __forceinline__ int ceil_log2(uint32_t L) { return L <= 1 ? 0 : 32 - 
 // Per-vertex mode (PV): matches are first aggregated in shared memory — per owner v in
 // ws.vcnt, per position of w in N+(u) at tc_smem[cbase + pos] — and flushed with one global
 // atomic per distinct vertex per item (hub vertices would otherwise serialise on atomics).
-template <bool PV, int S>
-__device__ __forceinline__ uint32_t wedge_loop(const uint32_t *__restrict__ col, const uint32_t *list, uint32_t sbase,
-                                               uint32_t cbase, uint32_t L, uint32_t lo, uint32_t hi, uint32_t total,
+template <bool PV, class Search>
+__device__ __forceinline__ uint32_t wedge_loop(const uint32_t *__restrict__ col, const Search &search, uint32_t sbase,
+                                               uint32_t cbase, uint32_t lo, uint32_t hi, uint32_t total,
                                                WarpScratch &ws, unsigned long long *tv) {
   uint32_t cnt = 0;
   uint32_t o = 0, o_beg = 0, o_end = ws.pre[0];
@@ -121,19 +168,12 @@ __device__ __forceinline__ uint32_t wedge_loop(const uint32_t *__restrict__ col,
 #pragma unroll
     for (int k = 0; k < UNR; ++k) {
       if (w[k] >= lo && w[k] <= hi) {
-        bool hit;
-        uint32_t pos = 0;
-        if (S > 0) {
-          pos = bsearch_pow2<S>(sbase, w[k]);
-          hit = tc_smem[pos] == w[k];
-        } else {
-          hit = bsearch_list(list, L, w[k]);
-        }
-        if (hit) {
+        uint32_t pos;
+        if (search(w[k], pos)) {
           ++cnt;
           if (PV) {
             atomicAdd(&ws.vcnt[ow[k]], 1u);
-            if (S > 0 && cbase != 0xffffffffu) atomicAdd(&tc_smem[cbase + (pos - sbase)], 1u);
+            if (cbase != 0xffffffffu) atomicAdd(&tc_smem[cbase + (pos - sbase)], 1u);
             else atomicAdd(&tv[w[k]], 1ull);
           }
         }
@@ -143,14 +183,37 @@ __device__ __forceinline__ uint32_t wedge_loop(const uint32_t *__restrict__ col,
   return cnt;
 }
 
+// Builds the bracket table of the staged list s = tc_smem[sbase .. sbase+L) (warp-wide):
+// tab[b] = first index whose bucket (s - lo) >> sh is >= b, b in [0, B]; returns
+// ceil(log2(max bucket occupancy)).
+__device__ __forceinline__ int build_bracket(uint32_t sbase, uint32_t tbase, uint32_t L, uint32_t lo, uint32_t hi,
+                                             uint32_t sh) {
+  const uint32_t B = ((hi - lo) >> sh) + 1;
+  uint16_t *tab = reinterpret_cast<uint16_t *>(tc_smem + tbase);
+  for (uint32_t j = lane_id(); j < L; j += 32) {
+    const uint32_t bj = (tc_smem[sbase + j] - lo) >> sh;
+    const int bp = j ? (int)((tc_smem[sbase + j - 1] - lo) >> sh) : -1;
+    for (int b = bp + 1; b <= (int)bj; ++b) tab[b] = (uint16_t)j;
+  }
+  if (lane_id() == 0) tab[B] = (uint16_t)L;
+  __syncwarp();
+  uint32_t mx = 0;
+  for (uint32_t b = lane_id(); b < B; b += 32) mx = max(mx, (uint32_t)tab[b + 1] - tab[b]);
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) mx = max(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+  return ceil_log2(mx);
+}
+
 // Count the wedges u->v->w of one chunk of up to 32 v's (lane-held `v`, `valid`) whose w
 // lies in list[0..L) (w restricted to [lo, hi]).  `padded`: list is the shared-memory copy
-// tc_smem[sbase ..] padded with +inf to 2^ceil(log2 L) entries.  Returns this lane's matches.
+// tc_smem[sbase ..] padded with +inf to 2^ceil(log2 L) (+64) entries; tbase != ~0: room
+// for a bracket table.  Returns this lane's matches.
 template <bool PV>
 __device__ __forceinline__ uint32_t warp_chunk(const uint64_t *__restrict__ offs, const uint32_t *__restrict__ col,
                                                uint32_t v, bool valid, const uint32_t *list, uint32_t sbase,
-                                               uint32_t cbase, uint32_t L, bool padded, uint32_t lo, uint32_t hi,
-                                               WarpScratch &ws, unsigned long long *tv) {
+                                               uint32_t tbase, uint32_t cbase, uint32_t L, bool padded, uint32_t lo,
+                                               uint32_t hi, WarpScratch &ws, unsigned long long *tv, int S2pre = -1,
+                                               uint32_t shpre = 0) {
   const unsigned lane = lane_id();
   uint64_t vb = 0;
   uint32_t dv = 0;
@@ -172,16 +235,31 @@ __device__ __forceinline__ uint32_t warp_chunk(const uint64_t *__restrict__ offs
   uint32_t cnt = 0;
   if (total) {
     const int S = padded ? ceil_log2(L) : 0;
-    switch (S) {
+    int S2 = S2pre >= 0 ? S2pre : 99;  // S2pre: table prebuilt by the CTA (large kernel)
+    uint32_t sh = shpre;
+    if (S2pre < 0 && S >= 6 && tbase != 0xffffffffu && g_bracket && total >= 2 * L) {
+      const int span_bits = 32 - __clz(hi - lo);  // bits of (hi - lo)
+      sh = span_bits > S ? (uint32_t)(span_bits - S) : 0u;
+      S2 = build_bracket(sbase, tbase, L, lo, hi, sh);
+      __syncwarp();
+    }
+    if (S2 <= 6) {
+      switch (S2) {
+#define TC_TAB(k) \
+  case k: cnt = wedge_loop<PV>(col, TabSearch<k>{sbase, tbase, lo, sh}, sbase, cbase, lo, hi, total, ws, tv); break;
+        TC_TAB(0) TC_TAB(1) TC_TAB(2) TC_TAB(3) TC_TAB(4) TC_TAB(5) TC_TAB(6)
+#undef TC_TAB
+      }
+    } else {
+      switch (S) {
 #define TC_CASE(k) \
-  case k:          \
-    cnt = wedge_loop<PV, k>(col, list, sbase, cbase, L, lo, hi, total, ws, tv); \
-    break;
-      TC_CASE(1) TC_CASE(2) TC_CASE(3) TC_CASE(4) TC_CASE(5) TC_CASE(6) TC_CASE(7)
-      TC_CASE(8) TC_CASE(9) TC_CASE(10) TC_CASE(11) TC_CASE(12) TC_CASE(13) TC_CASE(14)
+  case k: cnt = wedge_loop<PV>(col, Pow2Search<k>{sbase}, sbase, cbase, lo, hi, total, ws, tv); break;
+        TC_CASE(1) TC_CASE(2) TC_CASE(3) TC_CASE(4) TC_CASE(5) TC_CASE(6) TC_CASE(7)
+        TC_CASE(8) TC_CASE(9) TC_CASE(10) TC_CASE(11) TC_CASE(12) TC_CASE(13) TC_CASE(14)
 #undef TC_CASE
-      default:
-        cnt = wedge_loop<PV, 0>(col, list, sbase, cbase, L, lo, hi, total, ws, tv);
+        default:
+          cnt = wedge_loop<PV>(col, GlobalSearch{list, L}, sbase, 0xffffffffu, lo, hi, total, ws, tv);
+      }
     }
   }
   __syncwarp();
@@ -191,7 +269,8 @@ __device__ __forceinline__ uint32_t warp_chunk(const uint64_t *__restrict__ offs
 
 // One work item: source u, v's N+(u)[c0 .. c0+32) on one warp; N+(u) is searched in the
 // warp's shared slice (staged here, padded with +inf to a power of two) when it fits,
-// else in global memory.  PV: the slice is followed by cap match counters.
+// else in global memory.  Per-warp layout (warp_stride words): slice [cap + 64, +inf
+// padded], bracket table [cap + 64], PV only: match counters [cap].
 template <bool PV>
 __device__ __forceinline__ uint64_t warp_item(const uint64_t *__restrict__ offs, const uint32_t *__restrict__ col,
                                               uint32_t u, uint32_t c0, uint32_t sbase, uint32_t cap,
@@ -202,12 +281,12 @@ __device__ __forceinline__ uint64_t warp_item(const uint64_t *__restrict__ offs,
   if (L < 2 || c0 >= L) return 0;
   const uint32_t *list;
   bool padded = false;
-  const uint32_t cbase = (PV && L <= cap) ? sbase + cap : 0xffffffffu;
+  const uint32_t cbase = (PV && L <= cap) ? sbase + (cap + 64) + (cap + 64) / 2 : 0xffffffffu;
   if (L <= cap) {
-    const uint32_t P = 1u << ceil_log2(L);
+    const uint32_t P = (1u << ceil_log2(L)) + 64;
     for (uint32_t j = lane; j < P; j += 32) {
       tc_smem[sbase + j] = j < L ? ldg_u32(col + a + j) : 0xffffffffu;
-      if (PV) tc_smem[cbase + j] = 0;
+      if (PV && j < L) tc_smem[cbase + j] = 0;
     }
     __syncwarp();
     list = tc_smem + sbase;
@@ -218,7 +297,8 @@ __device__ __forceinline__ uint64_t warp_item(const uint64_t *__restrict__ offs,
   const uint32_t lo = list[0], hi = list[L - 1];
   const bool valid = c0 + lane < L;
   const uint32_t v = valid ? list[c0 + lane] : 0u;
-  uint32_t cnt = warp_chunk<PV>(offs, col, v, valid, list, sbase, cbase, L, padded, lo, hi, ws, tv);
+  uint32_t cnt = warp_chunk<PV>(offs, col, v, valid, list, sbase, padded ? sbase + cap + 64 : 0xffffffffu, cbase, L,
+                                padded, lo, hi, ws, tv);
   __syncwarp();  // slice reads done before the next item restages it
   if (PV) {
     uint64_t tot = warp_sum((uint64_t)cnt);
@@ -328,7 +408,7 @@ __global__ __launch_bounds__(CT_THREADS) void count_small_kernel(const uint64_t 
                                                                  uint64_t nheavy, unsigned long long *ctr, uint32_t cap,
                                                                  unsigned long long *T, unsigned long long *tv) {
   __shared__ WarpScratch s_ws[CT_WARPS];
-  const uint32_t slice = warp_id() * cap * (PV ? 2 : 1);  // PV: list + counters
+  const uint32_t slice = warp_id() * warp_stride(cap, PV);
   WarpScratch &ws = s_ws[warp_id()];
   uint64_t acc = 0;
   while (true) {  // heavy items, one per fetch
@@ -390,8 +470,10 @@ __global__ __launch_bounds__(LG_THREADS) void count_large_kernel(const uint64_t 
                                                                  const uint64_t *__restrict__ items, uint64_t nitems,
                                                                  unsigned long long *ctr, unsigned long long *T,
                                                                  unsigned long long *tv) {
-  uint32_t *s_piece = tc_smem;  // PIECE + 8 words (alignment slack)
+  uint32_t *s_piece = tc_smem;  // PIECE + 72 words (alignment slack + padding), then the table
+  constexpr uint32_t tbase_lg = PIECE + 72;
   __shared__ WarpScratch s_ws[LG_WARPS];
+  __shared__ uint32_t s_red[LG_WARPS];
   __shared__ __align__(8) uint64_t s_bar;
   __shared__ unsigned long long s_item;
   WarpScratch &ws = s_ws[warp_id()];
@@ -427,17 +509,45 @@ __global__ __launch_bounds__(LG_THREADS) void count_large_kernel(const uint64_t 
       mbar_wait(&s_bar, phase);
       phase ^= 1u;
       const uint32_t *list = s_piece + shift;
-      {  // pad the piece with +inf up to a power of two for the fixed-depth search
-        const uint32_t P = 1u << ceil_log2(plen);
+      {  // pad the piece with +inf up to a power of two (+64) for the fixed-depth search
+        const uint32_t P = (1u << ceil_log2(plen)) + 64;
         for (uint32_t j = plen + threadIdx.x; j < P; j += LG_THREADS) s_piece[shift + j] = 0xffffffffu;
         __syncthreads();
       }
       const uint32_t lo = list[0], hi = list[plen - 1];
+      // CTA-wide bracket table of the piece (shared by all warps of the item)
+      int S2 = -1;
+      uint32_t sh = 0;
+      const int S = ceil_log2(plen);
+      if (g_bracket && S >= 6) {
+        const int span_bits = 32 - __clz(hi - lo);
+        sh = span_bits > S ? (uint32_t)(span_bits - S) : 0u;
+        const uint32_t B = ((hi - lo) >> sh) + 1;
+        uint16_t *tab = reinterpret_cast<uint16_t *>(tc_smem + tbase_lg);
+        for (uint32_t j = threadIdx.x; j < plen; j += LG_THREADS) {
+          const uint32_t bj = (list[j] - lo) >> sh;
+          const int bp = j ? (int)((list[j - 1] - lo) >> sh) : -1;
+          for (int b = bp + 1; b <= (int)bj; ++b) tab[b] = (uint16_t)j;
+        }
+        if (threadIdx.x == 0) tab[B] = (uint16_t)plen;
+        __syncthreads();
+        uint32_t mx = 0;
+        for (uint32_t b = threadIdx.x; b < B; b += LG_THREADS) mx = max(mx, (uint32_t)tab[b + 1] - tab[b]);
+        mx = warp_max(mx);
+        if (lane_id() == 0) s_red[warp_id()] = mx;
+        __syncthreads();
+        mx = 0;
+        for (int w = 0; w < LG_WARPS; ++w) mx = max(mx, s_red[w]);
+        S2 = ceil_log2(mx);
+        if (S2 > 6) S2 = -1;  // pathological skew: plain fixed-depth search
+        __syncthreads();
+      }
       uint32_t cnt = 0;
       for (uint32_t c0 = cbeg + warp_id() * 32; c0 < cend; c0 += LG_THREADS) {
         bool valid = c0 + lane_id() < cend;
         uint32_t v = valid ? ldg_u32(col + a + c0 + lane_id()) : 0u;
-        cnt += warp_chunk<PV>(offs, col, v, valid, list, shift, 0xffffffffu, plen, true, lo, hi, ws, tv);
+        cnt += warp_chunk<PV>(offs, col, v, valid, list, shift, S2 >= 0 ? tbase_lg : 0xffffffffu, 0xffffffffu, plen,
+                              true, lo, hi, ws, tv, S2 >= 0 ? S2 : -2, sh);
       }
       ucnt += cnt;
       __syncthreads();  // piece fully consumed before the next bulk copy overwrites it
@@ -461,7 +571,7 @@ __global__ __launch_bounds__(CT_THREADS) void count_range_kernel(const uint64_t 
                                                                  unsigned long long *T, unsigned long long *tv) {
   __shared__ WarpScratch s_ws[CT_WARPS];
   __shared__ uint32_t s_bucket;
-  const uint32_t slice = warp_id() * cap * (PV ? 2 : 1);  // PV: list + counters
+  const uint32_t slice = warp_id() * warp_stride(cap, PV);
   WarpScratch &ws = s_ws[warp_id()];
   uint64_t acc = 0;
   while (true) {  // buckets fetched dynamically: a CTA takes the next bucket when done
@@ -544,7 +654,7 @@ __global__ void bounds_kernel(const uint64_t *__restrict__ pre, uint32_t n, uint
 static void configure_kernels() {
   static bool done = false;
   if (done) return;
-  size_t large_smem = (PIECE + 8) * sizeof(uint32_t);
+  size_t large_smem = LG_SMEM_WORDS * sizeof(uint32_t);
   TC_CUDA(cudaFuncSetAttribute(count_large_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)large_smem));
   TC_CUDA(cudaFuncSetAttribute(count_large_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)large_smem));
   int small_max = 200 * 1024;
@@ -604,6 +714,13 @@ static int occupancy(const void *fn, int threads, size_t smem) {
 uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *kernel_ms, uint64_t *launches) {
   cudaStream_t s = g.stream;
   configure_kernels();
+  {
+    static int last_bracket = 1;
+    if (g_opt_bracket != last_bracket) {
+      TC_CUDA(cudaMemcpyToSymbol(g_bracket, &g_opt_bracket, sizeof(int)));
+      last_bracket = g_opt_bracket;
+    }
+  }
   if (ue > g.n) ue = g.n;
   uint64_t nlaunch = 0;
   DevBuf<unsigned long long> dT;
@@ -641,7 +758,7 @@ uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *
         nb = (ue + k - 1) / k - b0;
       }
       if (nb) {
-        size_t smem = (size_t)CT_WARPS * cap * (tv ? 2 : 1) * sizeof(uint32_t);
+        size_t smem = (size_t)CT_WARPS * warp_stride(cap, tv != nullptr) * sizeof(uint32_t);
         int occ = occupancy(tv ? (const void *)count_range_kernel<true> : (const void *)count_range_kernel<false>,
                             CT_THREADS, smem);
         unsigned grid = (unsigned)std::min<uint64_t>(nb, (uint64_t)num_sms() * occ);
@@ -679,6 +796,14 @@ uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *
         if (b >= capbin) nlarge += hh[b];
         else if (b >= 5) nheavy += hh[b];  // d~ >= 32: fetched one item at a time
       }
+      // warp slices only as large as the longest warp-item list needs (occupancy: an ER
+      // graph with d~ < 32 gets 64-word slices, not 1024)
+      uint32_t cap_small = 32;
+      for (int b = capbin - 1; b >= 0; --b)
+        if (hh[b]) {
+          cap_small = std::max<uint32_t>(32, std::min<uint32_t>(cap, 1u << (b + 1)));
+          break;
+        }
       nlaunch += 2;
       if (nitems) {
         DevBuf<uint64_t> items;
@@ -692,7 +817,7 @@ uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *
         }
         if (kernel_ms) TC_CUDA(cudaEventRecord(e0, s));
         if (nlarge) {
-          size_t smem = (PIECE + 8) * sizeof(uint32_t);
+          size_t smem = LG_SMEM_WORDS * sizeof(uint32_t);
           int occ = occupancy(tv ? (const void *)count_large_kernel<true> : (const void *)count_large_kernel<false>,
                               LG_THREADS, smem);
           unsigned grid = (unsigned)std::min<uint64_t>(nlarge, (uint64_t)num_sms() * occ);
@@ -708,7 +833,7 @@ uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *
         }
         uint64_t nsmall = nitems - nlarge;
         if (nsmall) {
-          size_t smem = (size_t)CT_WARPS * cap * (tv ? 2 : 1) * sizeof(uint32_t);
+          size_t smem = (size_t)CT_WARPS * warp_stride(cap_small, tv != nullptr) * sizeof(uint32_t);
           int occ = occupancy(tv ? (const void *)count_small_kernel<true> : (const void *)count_small_kernel<false>,
                               CT_THREADS, smem);
           uint64_t want = (nsmall + CT_WARPS - 1) / CT_WARPS;
@@ -716,11 +841,12 @@ uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *
           ProfScope prof("count_small", s, 0.0);
           if (tv)
             count_small_kernel<true><<<grid, CT_THREADS, smem, s>>>(g.offs.get(), g.col.get(), items.get() + nlarge,
-                                                                     nsmall, nheavy, hist.get() + 65, cap, dT.get(), tv);
+                                                                     nsmall, nheavy, hist.get() + 65, cap_small,
+                                                                     dT.get(), tv);
           else
             count_small_kernel<false><<<grid, CT_THREADS, smem, s>>>(g.offs.get(), g.col.get(), items.get() + nlarge,
-                                                                      nsmall, nheavy, hist.get() + 65, cap, dT.get(),
-                                                                      nullptr);
+                                                                      nsmall, nheavy, hist.get() + 65, cap_small,
+                                                                      dT.get(), nullptr);
           TC_LAUNCH_CHECK();
           ++nlaunch;
         }

@@ -92,5 +92,6 @@ void analyze_graph(Graph &g);
 extern int g_opt_profile;
 extern int g_opt_small_cap;
 extern int g_opt_l2_persist;
+extern int g_opt_bracket;
 
 }  // namespace tc

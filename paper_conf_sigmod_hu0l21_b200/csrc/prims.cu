@@ -144,8 +144,19 @@ __global__ __launch_bounds__(T_THREADS) void rs_hist_kernel(Src keys, uint64_t n
   for (int i = threadIdx.x; i < groups * passes * 256; i += T_THREADS) s_h[i] = 0;
   __syncthreads();
   uint32_t *mine = s_h + (warp_id() / 2) * passes * 256;
-  uint64_t stride = (uint64_t)gridDim.x * T_THREADS;
-  for (uint64_t i = (uint64_t)blockIdx.x * T_THREADS + threadIdx.x; i < n; i += stride) {
+  // 8 independent loads in flight per thread before the shared-memory counting
+  constexpr int U = 8;
+  const uint64_t stride = (uint64_t)gridDim.x * T_THREADS;
+  uint64_t i = (uint64_t)blockIdx.x * T_THREADS + threadIdx.x;
+  for (; i + (U - 1) * stride < n; i += U * stride) {
+    uint64_t k[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u) k[u] = keys.load(i + u * stride);
+#pragma unroll
+    for (int u = 0; u < U; ++u)
+      for (int p = 0; p < passes; ++p) atomicAdd(&mine[p * 256 + ((k[u] >> (begin_bit + 8 * p)) & 255u)], 1u);
+  }
+  for (; i < n; i += stride) {
     uint64_t k = keys.load(i);
     for (int p = 0; p < passes; ++p) atomicAdd(&mine[p * 256 + ((k >> (begin_bit + 8 * p)) & 255u)], 1u);
   }
@@ -191,23 +202,48 @@ __device__ __forceinline__ uint32_t rank_item(uint32_t d, bool valid, uint32_t *
   return old + __popc(peers & lt_mask);
 }
 
+// Same rank with a shared-memory peer mask instead of 8 ballots: every lane ORs its bit
+// into mask[d]; after a warp barrier the mask IS the peer set.  The leader advances the
+// warp's counter and clears the mask (masks double-buffered across consecutive items so
+// the clear never races the next item's ORs).  ~12 instructions per key instead of ~30.
+__device__ __forceinline__ uint32_t rank_item_or(uint32_t d, bool valid, uint32_t *whist, uint32_t *mask,
+                                                 unsigned lane, unsigned lt_mask) {
+  if (valid) atomicOr(&mask[d], 1u << lane);
+  __syncwarp();
+  const unsigned peers = valid ? mask[d] : 0u;
+  __syncwarp();
+  uint32_t old = 0;
+  const unsigned lead = __ffs(peers) - 1;
+  if (valid && lane == lead) {
+    old = whist[d];
+    whist[d] = old + __popc(peers);
+    mask[d] = 0;
+  }
+  old = __shfl_sync(0xffffffffu, old, valid ? lead : lane);
+  return old + __popc(peers & lt_mask);
+}
+
 template <class Src>
-__global__ __launch_bounds__(T_THREADS, 3) void rs_pass_kernel(Src in, uint64_t *__restrict__ out, uint64_t n,
+__global__ __launch_bounds__(T_THREADS, 4) void rs_pass_kernel(Src in, uint64_t *__restrict__ out, uint64_t n,
                                                                int shift,
                                                                const unsigned long long *__restrict__ goff,
                                                                uint64_t *status, uint32_t *tile_ctr) {
   __shared__ uint64_t s_keys[T_TILE];
   __shared__ uint32_t s_whist[T_WARPS][256];
   __shared__ uint32_t s_cnt[256];
-  __shared__ uint32_t s_lstart[256];
   __shared__ uint64_t s_gbase[256];
   __shared__ uint32_t s_warp32[8];
   __shared__ uint32_t s_total32;
   __shared__ uint32_t s_tile;
   const unsigned w = warp_id(), l = lane_id(), t = threadIdx.x;
   if (t == 0) s_tile = atomicAdd(tile_ctr, 1u);
+  // ranking peer masks [2 buffers][warp][digit] alias the key staging area, which is only
+  // written after ranking completes
+  uint32_t *s_mask = reinterpret_cast<uint32_t *>(s_keys);
 #pragma unroll
   for (int i = 0; i < T_WARPS; ++i) s_whist[i][t] = 0;
+#pragma unroll
+  for (int i = 0; i < 2 * T_WARPS; ++i) s_mask[i * 256 + t] = 0;
   s_cnt[t] = 0;
   __syncthreads();
   const uint64_t tile = s_tile;
@@ -233,28 +269,25 @@ __global__ __launch_bounds__(T_THREADS, 3) void rs_pass_kernel(Src in, uint64_t 
   const uint32_t tcount = s_cnt[t];
   uint64_t *st = status + t;  // status laid out [tile][256]
   st_relaxed_u64(st + tile * 256, (tile == 0 ? LB_INC : LB_AGG) | tcount);
+  // tile-local start of digit t (known before ranking thanks to the early counts)
+  const uint32_t lstart = block256_exclusive_scan<uint32_t>(tcount, s_warp32, &s_total32);
 
   const unsigned lt_mask = (1u << l) - 1u;
   uint32_t *whist = s_whist[w];
-  if (full) {
+  uint32_t *mask0 = s_mask + w * 256, *mask1 = s_mask + (T_WARPS + w) * 256;
 #pragma unroll
-    for (int i = 0; i < T_ITEMS; ++i) r[i] = rank_item<true>((uint32_t)(k[i] >> shift) & 255u, true, whist, lt_mask);
-  } else {
-#pragma unroll
-    for (int i = 0; i < T_ITEMS; ++i)
-      r[i] = rank_item<false>((uint32_t)(k[i] >> shift) & 255u, wbase + i * 32 < n, whist, lt_mask);
-  }
+  for (int i = 0; i < T_ITEMS; ++i)
+    r[i] = rank_item_or((uint32_t)(k[i] >> shift) & 255u, full || wbase + i * 32 < n, whist, (i & 1) ? mask1 : mask0,
+                        l, lt_mask);
   __syncthreads();
-  // digit t: exclusive prefix over warps
-  uint32_t run = 0;
+  // digit t: tile-local start + exclusive prefix over warps -> per-warp scatter base
+  uint32_t run = lstart;
 #pragma unroll
   for (int ww = 0; ww < T_WARPS; ++ww) {
     uint32_t c = s_whist[ww][t];
     s_whist[ww][t] = run;
     run += c;
   }
-  uint32_t lstart = block256_exclusive_scan<uint32_t>(tcount, s_warp32, &s_total32);
-  s_lstart[t] = lstart;
   // look-back for digit t, four predecessors per round trip
   uint64_t e = 0;
   if (tile > 0) {
@@ -279,19 +312,26 @@ __global__ __launch_bounds__(T_THREADS, 3) void rs_pass_kernel(Src in, uint64_t 
     }
     st_relaxed_u64(st + tile * 256, LB_INC | (e + tcount));
   }
-  s_gbase[t] = goff[t] + e;
+  s_gbase[t] = goff[t] + e - lstart;  // global position of tile slot j of digit t = s_gbase[t] + j
   __syncthreads();
 #pragma unroll
   for (int i = 0; i < T_ITEMS; ++i) {
     uint32_t d = (uint32_t)(k[i] >> shift) & 255u;
-    if (full || wbase + i * 32 < n) s_keys[s_lstart[d] + s_whist[w][d] + r[i]] = k[i];
+    if (full || wbase + i * 32 < n) s_keys[s_whist[w][d] + r[i]] = k[i];
   }
   __syncthreads();
-  uint64_t valid_count = n - base < (uint64_t)T_TILE ? n - base : (uint64_t)T_TILE;
-  for (uint32_t j = t; j < valid_count; j += T_THREADS) {
-    uint64_t key = s_keys[j];
-    uint32_t dd = (uint32_t)((key >> shift) & 255u);
-    out[s_gbase[dd] + j - s_lstart[dd]] = key;
+  if (full) {
+#pragma unroll 4
+    for (uint32_t j = t; j < T_TILE; j += T_THREADS) {
+      uint64_t key = s_keys[j];
+      out[s_gbase[(uint32_t)(key >> shift) & 255u] + j] = key;
+    }
+  } else {
+    const uint32_t valid_count = (uint32_t)(n - base);
+    for (uint32_t j = t; j < valid_count; j += T_THREADS) {
+      uint64_t key = s_keys[j];
+      out[s_gbase[(uint32_t)(key >> shift) & 255u] + j] = key;
+    }
   }
 }
 

@@ -99,7 +99,7 @@ def test_config1_rmat_s16(d, r):
 
 
 @pytest.mark.parametrize("sched", ["bucketed", "range"])
-@pytest.mark.parametrize("cap", [32, 64, 1024])
+@pytest.mark.parametrize("cap", [32, 64, 256, 2048])
 def test_schedules_and_caps(sched, cap):
     """Every kernel path (warp slice, global-search fallback, CTA+TMA pieces) counts the same."""
     spec = graphgen.rmat_spec(13, 16, 77)
@@ -113,11 +113,11 @@ def test_schedules_and_caps(sched, cap):
             assert T == ref["T"] and np.array_equal(t, ref["t"])
             g.free()
     finally:
-        tc.tc_set_option("small_cap", 1024)
+        tc.tc_set_option("small_cap", 256)
 
 
 def test_large_kernel_multi_piece():
-    """A star-heavy graph with ID directing: one source list > PIECE (16384) elements."""
+    """A star-heavy graph with ID directing: one source list spans several TMA pieces."""
     rng = np.random.default_rng(9)
     n = 40000
     hub = 0
