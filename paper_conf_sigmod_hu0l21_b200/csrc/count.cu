@@ -283,7 +283,8 @@ __device__ __forceinline__ uint64_t warp_item(const uint64_t *__restrict__ offs,
   bool padded = false;
   const uint32_t cbase = (PV && L <= cap) ? sbase + (cap + 64) + (cap + 64) / 2 : 0xffffffffu;
   if (L <= cap) {
-    const uint32_t P = (1u << ceil_log2(L)) + 64;
+    const int SL = ceil_log2(L);
+    const uint32_t P = (1u << SL) + (SL >= 6 ? 64u : 0u);  // +64: bracket-search slack
     for (uint32_t j = lane; j < P; j += 32) {
       tc_smem[sbase + j] = j < L ? ldg_u32(col + a + j) : 0xffffffffu;
       if (PV && j < L) tc_smem[cbase + j] = 0;
