@@ -191,7 +191,9 @@ def main():
     r = args.reorder or CONFIG_RULES[cfg][1]
     torch.cuda.set_device(local_rank)
     dev = torch.device("cuda", local_rank)
-    if world > 1:
+    # under torchrun (even with one rank) the count goes through tc_count_dist + NCCL
+    distributed = world > 1 or "LOCAL_RANK" in os.environ
+    if distributed:
         dist.init_process_group("nccl", device_id=dev)
     stream = torch.cuda.current_stream(dev)
     sptr = stream.cuda_stream
@@ -207,7 +209,7 @@ def main():
         flush = torch.empty(2 * L2_BYTES // 4, dtype=torch.int32, device=dev)
 
     comm = None
-    if world > 1:
+    if distributed:
         comm = tdist.init_nccl_comm(rank, world, local_rank)
 
     prm, keep = tc.make_aorder_params()
@@ -239,7 +241,7 @@ def main():
     # ---------------------------------------------------------------- timed region
     tc.tc_set_option("kernel_profile", 1)
     tc.tc_profile_report(reset=True)
-    if world > 1:
+    if distributed:
         dist.barrier()
     torch.cuda.synchronize()
     clocks = ClockSampler(local_rank)
@@ -259,7 +261,7 @@ def main():
             flush.fill_(1)
         times.append((e0, e1))
     torch.cuda.synchronize()
-    if world > 1:
+    if distributed:
         dist.barrier()
     clk = clocks.stop()
     tc.tc_set_option("kernel_profile", 0)
@@ -330,7 +332,7 @@ def main():
         hd.copy_(dst)
         step(hs, hd)
         torch.cuda.synchronize()
-        if world > 1:
+        if distributed:
             dist.barrier()
         ev = []
         for _ in range(args.steps):
@@ -359,7 +361,7 @@ def main():
     del keep
     if rank == 0:
         print(json.dumps(line), flush=True)
-    if world > 1:
+    if distributed:
         dist.barrier()
         dist.destroy_process_group()
 

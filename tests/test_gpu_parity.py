@@ -248,3 +248,39 @@ def test_gpu_generator_matches_cpu():
         cs, cd = graphgen.generate_cpu(spec)
         assert np.array_equal(s.cpu().numpy().view(np.uint32), cs)
         assert np.array_equal(d.cpu().numpy().view(np.uint32), cd)
+
+
+def test_count_dist_single_rank_nccl():
+    """a11 through the real NCCL path on one GPU: unique id, comm init, the slice count and
+    the ncclAllReduce of the uint64 partial (and of the per-vertex vector)."""
+    spec = graphgen.rmat_spec(13, 16, 21)
+    src, dst = graphgen.generate_cpu(spec)
+    ref = oracle.run(src, dst, spec.n, "paper", "paper", per_vertex=True)
+    uid = tc.tc_nccl_get_unique_id()
+    comm = tc.tc_nccl_comm_init(uid, 0, 1, 0)
+    try:
+        g = tc.Graph(src, dst, spec.n).direct("paper").reorder("paper")
+        assert tc.tc_count_dist(g.handle, comm, 0, 1) == ref["T"]
+        t = np.zeros(spec.n, np.uint64)
+        assert tc.tc_count_dist(g.handle, comm, 0, 1, t) == ref["T"]
+        assert np.array_equal(t, ref["t"])
+        g.free()
+    finally:
+        tc.tc_nccl_comm_destroy(comm)
+
+
+def test_bench_under_torchrun_single_process():
+    """bench.py's N>1 code path (torch.distributed NCCL + library comm) with one rank."""
+    import json
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "1",
+           "--master-addr", "127.0.0.1", "--master-port", "29533", os.path.join(root, "bench.py"),
+           "--gpus", "1", "--steps", "2", "--warmup", "1", "--config", "1", "--no-e2e", "--no-cpu-baseline"]
+    env = dict(os.environ, WORLD_SIZE="1")
+    out = subprocess.run(cmd, capture_output=True, text=True, timeout=600, env=env, cwd=root)
+    assert out.returncode == 0, out.stderr[-2000:]
+    line = json.loads(out.stdout.strip().splitlines()[-1])
+    assert line["config"]["triangles"] > 0 and line["value"] > 0
