@@ -35,12 +35,23 @@ __global__ void copy_deg_kernel(const uint32_t *__restrict__ deg, uint64_t *__re
 
 __global__ void sym_fill_kernel(const uint64_t *__restrict__ edges, uint64_t m, int bits,
                                 unsigned long long *__restrict__ cursor, uint32_t *__restrict__ adj) {
-  uint64_t mask = (1ull << bits) - 1;
-  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < m; i += (uint64_t)gridDim.x * blockDim.x) {
-    uint64_t k = edges[i];
-    uint32_t u = (uint32_t)(k >> bits), v = (uint32_t)(k & mask);
-    adj[atomicAdd(&cursor[u], 1ull)] = v;
-    adj[atomicAdd(&cursor[v], 1ull)] = u;
+  const uint64_t mask = (1ull << bits) - 1;
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  // edges are sorted by u: lanes sharing u reserve their slots with ONE atomic per run
+  for (uint64_t base = (uint64_t)blockIdx.x * blockDim.x + (threadIdx.x & ~31u); base < m; base += stride) {
+    const uint64_t i = base + lane_id();
+    const bool valid = i < m;
+    const uint64_t k = valid ? edges[i] : 0;
+    const uint32_t u = valid ? (uint32_t)(k >> bits) : 0xffffffffu, v = (uint32_t)(k & mask);
+    const unsigned peers = __match_any_sync(0xffffffffu, u);
+    const unsigned lead = __ffs(peers) - 1;
+    unsigned long long pu = 0;
+    if (valid && lane_id() == lead) pu = atomicAdd(&cursor[u], (unsigned long long)__popc(peers));
+    pu = __shfl_sync(0xffffffffu, pu, lead) + __popc(peers & ((1u << lane_id()) - 1u));
+    if (valid) {
+      adj[pu] = v;
+      adj[atomicAdd(&cursor[v], 1ull)] = u;
+    }
   }
 }
 
@@ -181,8 +192,9 @@ void peel_paper(Graph &g) {
   g.dsnap.alloc(n ? n : 1, s);
   TC_CUDA(cudaMemcpyAsync(res.get(), g.deg.get(), sizeof(uint32_t) * n, cudaMemcpyDeviceToDevice, s));
   TC_CUDA(cudaMemsetAsync(state.get(), 0, n, s));
-  unsigned *h_cnt = nullptr;
-  TC_CUDA(cudaMallocHost(&h_cnt, 2 * sizeof(unsigned)));
+  // pinned frontier counters, allocated once per host thread (cudaMallocHost is slow)
+  static thread_local unsigned *h_cnt = nullptr;
+  if (!h_cnt) TC_CUDA(cudaMallocHost(&h_cnt, 2 * sizeof(unsigned)));
   uint64_t peeled = 0;
   uint32_t level = 0, r = 0;
   ProfScope prof("peel", s, 0.0);
@@ -218,10 +230,8 @@ void peel_paper(Graph &g) {
       TC_REQUIRE(level < 200, ST_CUDA, "A-direction did not terminate");
     }
   } catch (...) {
-    cudaFreeHost(h_cnt);
     throw;
   }
-  cudaFreeHost(h_cnt);
   g.levels = level;
   g.subrounds = r;
   prim_paper_kernel<<<grid_for(n, 256), 256, 0, s>>>(g.sub.get(), g.dsnap.get(), g.prim.get(), n);
