@@ -9,7 +9,7 @@ OUT=gpurun_out
 mkdir -p $OUT
 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $OUT/launches_cfg${CFG}.csv \
     python bench.py --config $CFG --steps 2 --warmup 1 --no-e2e --no-cpu-baseline > $OUT/launches_bench.log 2>&1
-for K in rs_pass count_small count_large count_range unique_kernel rs_hist; do
+for K in rs_pass_kernel count_small count_large count_range unique_kernel rs_hist_kernel; do
   ncu --set full --clock-control none --import-source on -k regex:$K -s 1 -c 1 -o $OUT/full_cfg${CFG}_$K \
       python tools/timeline.py $CFG > /dev/null 2>&1 || true
 done

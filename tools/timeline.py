@@ -18,7 +18,8 @@ import os
 for kv in filter(None, os.environ.get("TC_OPTS", "").split(",")):
     k, v = kv.split("=")
     tc.tc_set_option(k, int(v))
-for it in range(4):
+ITERS = int(os.environ.get("ITERS", "4"))
+for it in range(ITERS):
     tc.tc_set_option("kernel_profile", 1)
     tc.tc_profile_report(reset=True)
     t = {}
@@ -31,7 +32,7 @@ for it in range(4):
     st = tc.tc_get_stats(g)
     t0 = time.perf_counter(); tc.tc_graph_free(g); t["free"] = time.perf_counter() - t0
     prof = tc.tc_profile_report(reset=True)
-    if it == 3:
+    if it == ITERS - 1:
         print("wall ms:", {k: round(v * 1e3, 3) for k, v in t.items()}, "total", round(sum(t.values()) * 1e3, 3))
         print("stage ms:", {k: round(st[k], 3) for k in ("ms_build", "ms_direct", "ms_reorder", "ms_count", "ms_count_kernel")})
         launches = prof.pop("_launches")
