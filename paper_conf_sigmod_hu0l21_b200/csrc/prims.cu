@@ -288,27 +288,38 @@ __global__ __launch_bounds__(T_THREADS, 4) void rs_pass_kernel(Src in, uint64_t 
     s_whist[ww][t] = run;
     run += c;
   }
-  // look-back for digit t, four predecessors per round trip
+  // look-back for digit t, four predecessors per round trip; flags tested on the high
+  // word, 32-bit bookkeeping (the walk is executed by every thread, so its instruction
+  // count matters as much as its round trips)
   uint64_t e = 0;
   if (tile > 0) {
-    int64_t j = (int64_t)tile - 1;
+    const uint64_t *p = st + (tile - 1) * 256;  // this digit's word of the newest predecessor
+    uint32_t left = (uint32_t)tile;             // predecessors not yet examined (p is valid)
     while (true) {
-      uint64_t v[4];
-#pragma unroll
-      for (int q = 0; q < 4; ++q) v[q] = (j - q >= 0) ? ld_relaxed_u64(st + (uint64_t)(j - q) * 256) : 0ull;
-      int q = 0;
-      bool done = false;
-#pragma unroll
-      for (int qq = 0; qq < 4; ++qq) {
-        if (done || q != qq || j - qq < 0) continue;
-        uint64_t f = v[qq] & ~LB_VAL;
-        if (f == 0) continue;
-        e += v[qq] & LB_VAL;
-        if (f == LB_INC) done = true;
-        else q = qq + 1;
+      const uint64_t v0 = ld_relaxed_u64(p);
+      const uint64_t v1 = left > 1 ? ld_relaxed_u64(p - 256) : 0ull;
+      const uint64_t v2 = left > 2 ? ld_relaxed_u64(p - 512) : 0ull;
+      const uint64_t v3 = left > 3 ? ld_relaxed_u64(p - 768) : 0ull;
+      const uint32_t h0 = (uint32_t)(v0 >> 32), h1 = (uint32_t)(v1 >> 32), h2 = (uint32_t)(v2 >> 32),
+                     h3 = (uint32_t)(v3 >> 32);
+      // flag (top two bits): 0 not out, 1 aggregate, 2 inclusive
+      if (h0 < 0x40000000u) {
+        __nanosleep(32);
+        continue;
       }
-      if (done) break;
-      j -= q;
+      e += v0 & LB_VAL;
+      if (h0 >= 0x80000000u) break;
+      if (h1 < 0x40000000u) { p -= 256; left -= 1; continue; }
+      e += v1 & LB_VAL;
+      if (h1 >= 0x80000000u) break;
+      if (h2 < 0x40000000u) { p -= 512; left -= 2; continue; }
+      e += v2 & LB_VAL;
+      if (h2 >= 0x80000000u) break;
+      if (h3 < 0x40000000u) { p -= 768; left -= 3; continue; }
+      e += v3 & LB_VAL;
+      if (h3 >= 0x80000000u) break;
+      p -= 1024;
+      left -= 4;
     }
     st_relaxed_u64(st + tile * 256, LB_INC | (e + tcount));
   }
