@@ -78,59 +78,118 @@ __global__ __launch_bounds__(T_THREADS) void scan_kernel(const TI *__restrict__ 
 }
 
 // ------------------------------------------------------------------ unique
+// Warp-wide decoupled look-back over one status word per tile (flag | value): lane i
+// examines predecessor tile - 1 - i, so one round trip covers 32 tiles.  Called by one
+// whole warp; returns the exclusive prefix of `tile` (all lanes) and publishes its
+// inclusive value.
+__device__ __forceinline__ uint64_t warp_lookback(uint64_t *status, uint64_t tile, uint64_t local) {
+  const unsigned l = lane_id();
+  if (tile == 0) {
+    if (l == 0) st_relaxed_u64(status, LB_INC | local);
+    return 0;
+  }
+  if (l == 0) st_relaxed_u64(status + tile, LB_AGG | local);
+  uint64_t excl = 0;
+  int64_t j = (int64_t)tile - 1;
+  while (true) {
+    const uint64_t v = (j - (int64_t)l >= 0) ? ld_relaxed_u64(status + (j - l)) : LB_INC;
+    const uint32_t h = (uint32_t)(v >> 32);
+    const unsigned notready = __ballot_sync(0xffffffffu, h < 0x40000000u);
+    const unsigned incm = __ballot_sync(0xffffffffu, h >= 0x80000000u);
+    const int lim = incm ? __ffs(incm) - 1 : 32;  // nearest inclusive value
+    const unsigned below = lim == 32 ? 0xffffffffu : ((1u << lim) - 1u);
+    if (notready & (below | (incm ? (1u << lim) : 0u))) {
+      __nanosleep(32);
+      continue;
+    }
+    excl += warp_sum((int)l <= lim ? (v & LB_VAL) : 0ull);
+    if (incm) break;
+    j -= 32;
+  }
+  if (l == 0) st_relaxed_u64(status + tile, LB_INC | (excl + local));
+  return excl;
+}
+
 // Unique-select; optionally (deg != nullptr) the undirected degrees of the kept edges
 // (step a3 fused): keys are (u << bits) | v, u < v; the sentinel key is dropped from deg.
+// Warp w of a tile owns 512 consecutive keys, lane l item i = key w*512 + 32*i + l
+// (coalesced loads and stores); the predecessor of a key comes from the neighbouring lane.
+// deg[v] takes one atomic per kept key; deg[u] one per run of equal u within a 32-key row.
 __global__ __launch_bounds__(T_THREADS) void unique_kernel(const uint64_t *__restrict__ in,
                                                            uint64_t *__restrict__ out, uint64_t n,
                                                            uint64_t *status, uint32_t *tile_ctr,
                                                            uint64_t ntiles, uint64_t *d_count, uint32_t *deg,
                                                            int bits, uint64_t sentinel) {
-  __shared__ uint64_t s_warp[8];
-  __shared__ uint64_t s_total;
+  __shared__ uint32_t s_wcnt[T_WARPS];
+  __shared__ uint64_t s_base;
   __shared__ uint32_t s_tile;
-  __shared__ uint64_t s_excl;
   if (threadIdx.x == 0) s_tile = atomicAdd(tile_ctr, 1u);
   __syncthreads();
-  uint64_t tile = s_tile;
-  uint64_t base = tile * T_TILE + (uint64_t)threadIdx.x * T_ITEMS;
+  const uint64_t tile = s_tile;
+  const unsigned w = warp_id(), l = lane_id();
+  const uint64_t wb = tile * T_TILE + (uint64_t)w * (32 * T_ITEMS);
   uint64_t k[T_ITEMS];
-  uint32_t flags = 0;
-  uint64_t prev = (base > 0 && base <= n) ? in[base - 1] : 0;
+  unsigned hm[T_ITEMS];
+  uint64_t before = 0;
+  if (l == 0 && wb > 0 && wb <= n) before = in[wb - 1];
 #pragma unroll
   for (int i = 0; i < T_ITEMS; ++i) {
-    uint64_t idx = base + i;
-    k[i] = idx < n ? in[idx] : 0;
-    bool head = idx < n && (idx == 0 || k[i] != prev);
-    flags |= (uint32_t)head << i;
-    prev = k[i];
+    const uint64_t idx = wb + 32 * i + l;
+    k[i] = idx < n ? __ldcs(in + idx) : 0ull;
   }
-  uint64_t cnt = __popc(flags);
-  uint64_t excl_t = block256_exclusive_scan<uint64_t>(cnt, s_warp, &s_total);
-  if (threadIdx.x == 0) {
-    s_excl = lookback_exclusive(status, tile, 1, s_total);
-    if (tile == ntiles - 1) *d_count = s_excl + s_total;
+  uint32_t wcnt = 0;
+#pragma unroll
+  for (int i = 0; i < T_ITEMS; ++i) {
+    const uint64_t idx = wb + 32 * i + l;
+    uint64_t prev = __shfl_up_sync(0xffffffffu, k[i], 1);
+    const uint64_t last_prev_row = __shfl_sync(0xffffffffu, i ? k[i - 1] : before, 31);
+    if (l == 0) prev = i ? last_prev_row : before;
+    const bool head = idx < n && (idx == 0 || k[i] != prev);
+    hm[i] = __ballot_sync(0xffffffffu, head);
+    wcnt += __popc(hm[i]);
+  }
+  if (l == 0) s_wcnt[w] = wcnt;
+  __syncthreads();
+  if (w == 0) {
+    const uint32_t c = l < T_WARPS ? s_wcnt[l] : 0u;
+    const uint32_t inc = warp_inclusive_scan(c);
+    const uint32_t total = __shfl_sync(0xffffffffu, inc, 31);
+    const uint64_t excl = warp_lookback(status, tile, total);
+    if (l < T_WARPS) s_wcnt[l] = inc - c;
+    if (l == 0) {
+      s_base = excl;
+      if (tile == ntiles - 1) *d_count = excl + total;
+    }
   }
   __syncthreads();
-  uint64_t pos = s_excl + excl_t;
+  uint64_t pos = s_base + s_wcnt[w];
+  const unsigned lt = (1u << l) - 1u;
 #pragma unroll
-  for (int i = 0; i < T_ITEMS; ++i)
-    if (flags >> i & 1u) out[pos++] = k[i];
+  for (int i = 0; i < T_ITEMS; ++i) {
+    if (hm[i] >> l & 1u) out[pos + __popc(hm[i] & lt)] = k[i];
+    pos += __popc(hm[i]);
+  }
   if (deg) {
     const uint64_t mask = (1ull << bits) - 1;
-    uint32_t ru = 0xffffffffu, rc = 0;  // run of equal u among this thread's heads
 #pragma unroll
     for (int i = 0; i < T_ITEMS; ++i) {
-      if (!(flags >> i & 1u) || k[i] == sentinel) continue;
-      uint32_t u = (uint32_t)(k[i] >> bits), v = (uint32_t)(k[i] & mask);
-      atomicAdd(&deg[v], 1u);
-      if (u != ru) {
-        if (rc) atomicAdd(&deg[ru], rc);
-        ru = u;
-        rc = 0;
+      const bool keep = (hm[i] >> l & 1u) && k[i] != sentinel;
+      const uint32_t u = (uint32_t)(k[i] >> bits), v = (uint32_t)(k[i] & mask);
+      if (keep) atomicAdd(&deg[v], 1u);
+      // runs of equal u along the row (keys ascending): the run's last lane adds its kept count
+      const unsigned km = __ballot_sync(0xffffffffu, keep);
+      if (!km) continue;
+      const uint32_t un = __shfl_down_sync(0xffffffffu, u, 1);
+      const uint32_t up = __shfl_up_sync(0xffffffffu, u, 1);
+      const unsigned starts = __ballot_sync(0xffffffffu, l == 0 || up != u);
+      const bool last = l == 31 || un != u;
+      if (last) {
+        const unsigned upto = l == 31 ? 0xffffffffu : ((2u << l) - 1u);
+        const int rs = 31 - __clz(starts & upto);
+        const unsigned c = __popc(km & upto & ~((1u << rs) - 1u));
+        if (c) atomicAdd(&deg[u], c);
       }
-      ++rc;
     }
-    if (rc) atomicAdd(&deg[ru], rc);
   }
 }
 
