@@ -166,8 +166,10 @@ tc_status tc_export_buckets(tc_graph *g, uint32_t *bucket_off);
  * "kernel_profile" (0/1: per-kernel event pairs for tc_profile_report, default 0),
  * "small_cap" (power of two in [32, 2048]; d~(u) below it is counted with N+(u) in a
  * per-warp shared-memory slice, default 256), "l2_persist" (0/1: L2 access-policy window
- * over the CSR during counts, default 0), "trim_memory" (any value: release the library's
- * cached device blocks). */
+ * over the CSR during counts, default 0), "split" (0/1: with original labels, build the
+ * oriented CSR by splitting the sorted edge list into forward and reversed runs and sorting
+ * only the reversed run, default 1; 0 = sort every oriented key), "trim_memory" (any
+ * value: release the library's cached device blocks). */
 tc_status tc_set_option(const char *key, int64_t value);
 
 /* Per-kernel profile since the last reset, as JSON text into buf (host, cap bytes):

@@ -76,20 +76,89 @@ __global__ void frontier_init_kernel(const uint8_t *__restrict__ state, const ui
   }
 }
 
+// Marks the frontier (snapshot at formation) and splits it by degree for the three expand
+// kernels: d(v) <= 32 -> Fs (flattened, 32 vertices per warp), 32 < d(v) <= HUGE_DEG -> Fb
+// (warp per vertex), d(v) > HUGE_DEG -> Fh (the whole grid per vertex: a hub never
+// serialises on one warp).  Vertices with d(v) = 0 have nothing to expand.
+constexpr uint32_t HUGE_DEG = 4096;
 __global__ void mark_kernel(const uint32_t *__restrict__ F, unsigned nf, uint8_t *state,
-                            const uint32_t *__restrict__ res, uint32_t *sub, uint32_t *dsnap, uint32_t r) {
-  for (unsigned i = blockIdx.x * blockDim.x + threadIdx.x; i < nf; i += gridDim.x * blockDim.x) {
-    uint32_t v = F[i];
-    state[v] = V_FRONTIER;
-    sub[v] = r;
-    dsnap[v] = res[v];
+                            const uint32_t *__restrict__ res, const uint32_t *__restrict__ deg, uint32_t *sub,
+                            uint32_t *dsnap, uint32_t r, uint32_t *Fs, uint32_t *Fb, uint32_t *Fh,
+                            unsigned *cnt_sb) {
+  for (unsigned base = blockIdx.x * blockDim.x + (threadIdx.x & ~31u); base < nf; base += gridDim.x * blockDim.x) {
+    const unsigned i = base + lane_id();
+    uint32_t v = 0, d = 0;
+    if (i < nf) {
+      v = F[i];
+      state[v] = V_FRONTIER;
+      sub[v] = r;
+      dsnap[v] = res[v];
+      d = deg[v];
+    }
+    warp_append(i < nf && d != 0 && d <= 32, v, Fs, cnt_sb);
+    warp_append(i < nf && d > 32 && d <= HUGE_DEG, v, Fb, cnt_sb + 1);
+    warp_append(i < nf && d > HUGE_DEG, v, Fh, cnt_sb + 2);
   }
 }
 
-// One warp per frontier vertex; lanes stride over N(v).
-__global__ void expand_kernel(const uint32_t *__restrict__ F, unsigned nf, const uint64_t *__restrict__ soffs,
+// Decrement of one incident edge (v, nbr) of a frontier vertex (Algorithm 1 line 12-16).
+__device__ __forceinline__ bool expand_one(uint32_t nbr, const uint8_t *__restrict__ state, uint32_t *res,
+                                           uint64_t thr) {
+  if (state[nbr] != V_UNPEELED) return false;
+  const uint32_t old = atomicSub(&res[nbr], 1u);
+  return (uint64_t)old == thr + 1;
+}
+
+// Frontier vertices with d(v) <= 32, 32 per warp: their adjacency lists are flattened
+// (warp inclusive scan of the degrees) so every lane handles one incident edge per step;
+// the owner of flattened element j is found by a 5-step search over the scan in registers.
+__global__ void expand_flat_kernel(const uint32_t *__restrict__ F, const unsigned *__restrict__ nfp,
+                                   const uint64_t *__restrict__ soffs, const uint32_t *__restrict__ sadj,
+                                   const uint8_t *__restrict__ state, uint32_t *res, uint64_t thr, uint32_t *next,
+                                   unsigned *nnext) {
+  const unsigned nf = *nfp;
+  const unsigned warps = gridDim.x * (blockDim.x / 32);
+  const unsigned lane = lane_id();
+  for (unsigned g0 = (blockIdx.x * (blockDim.x / 32) + warp_id()) * 32; g0 < nf; g0 += warps * 32) {
+    uint64_t a = 0;
+    uint32_t d = 0;
+    if (g0 + lane < nf) {
+      const uint32_t v = F[g0 + lane];
+      a = soffs[v];
+      d = (uint32_t)(soffs[v + 1] - a);
+    }
+    const uint32_t inc = warp_inclusive_scan(d);
+    const uint32_t total = __shfl_sync(0xffffffffu, inc, 31);
+    for (uint32_t j0 = 0; j0 < total; j0 += 32) {
+      const uint32_t j = j0 + lane;
+      // owner o = number of lanes whose inclusive prefix is <= j (binary search over lanes)
+      uint32_t o = 0;
+#pragma unroll
+      for (int k = 4; k >= 0; --k) {
+        const uint32_t q = o + (1u << k);
+        const uint32_t pq = __shfl_sync(0xffffffffu, inc, (q - 1) & 31);
+        if (q <= 32 && pq <= j) o = q;
+      }
+      const uint32_t oo = o & 31;
+      const uint64_t ao = __shfl_sync(0xffffffffu, a, oo);
+      const uint32_t eo = __shfl_sync(0xffffffffu, inc, oo) - __shfl_sync(0xffffffffu, d, oo);
+      bool cross = false;
+      uint32_t nbr = 0;
+      if (j < total) {
+        nbr = sadj[ao + (j - eo)];
+        cross = expand_one(nbr, state, res, thr);
+      }
+      warp_append(cross, nbr, next, nnext);
+    }
+  }
+}
+
+// Frontier vertices with d(v) > 32: one warp per vertex; lanes stride over N(v).
+__global__ void expand_kernel(const uint32_t *__restrict__ F, const unsigned *__restrict__ nfp,
+                              const uint64_t *__restrict__ soffs,
                               const uint32_t *__restrict__ sadj, const uint8_t *__restrict__ state,
                               uint32_t *res, uint64_t thr, uint32_t *next, unsigned *nnext) {
+  const unsigned nf = *nfp;
   unsigned warps = gridDim.x * (blockDim.x / 32);
   for (unsigned i = blockIdx.x * (blockDim.x / 32) + warp_id(); i < nf; i += warps) {
     uint32_t v = F[i];
@@ -100,10 +169,32 @@ __global__ void expand_kernel(const uint32_t *__restrict__ F, unsigned nf, const
       uint32_t nbr = 0;
       if (p < e) {
         nbr = sadj[p];
-        if (state[nbr] == V_UNPEELED) {
-          uint32_t old = atomicSub(&res[nbr], 1u);
-          cross = (uint64_t)old == thr + 1;
-        }
+        cross = expand_one(nbr, state, res, thr);
+      }
+      warp_append(cross, nbr, next, nnext);
+    }
+  }
+}
+
+// Frontier hubs (d(v) > HUGE_DEG), one after another, each spread over every thread of
+// the grid; the appends stay warp-aggregated.
+__global__ void expand_huge_kernel(const uint32_t *__restrict__ F, const unsigned *__restrict__ nfp,
+                                   const uint64_t *__restrict__ soffs, const uint32_t *__restrict__ sadj,
+                                   const uint8_t *__restrict__ state, uint32_t *res, uint64_t thr, uint32_t *next,
+                                   unsigned *nnext) {
+  const unsigned nf = *nfp;
+  const uint64_t nthreads = (uint64_t)gridDim.x * blockDim.x;
+  const uint64_t tid0 = (uint64_t)blockIdx.x * blockDim.x + (threadIdx.x & ~31u);
+  for (unsigned i = 0; i < nf; ++i) {
+    const uint32_t v = F[i];
+    const uint64_t a = soffs[v], e = soffs[v + 1];
+    for (uint64_t p0 = a + tid0; p0 < e; p0 += nthreads) {
+      const uint64_t p = p0 + lane_id();
+      bool cross = false;
+      uint32_t nbr = 0;
+      if (p < e) {
+        nbr = sadj[p];
+        cross = expand_one(nbr, state, res, thr);
       }
       warp_append(cross, nbr, next, nnext);
     }
@@ -180,14 +271,17 @@ void peel_paper(Graph &g) {
       TC_LAUNCH_CHECK();
     }
   }
-  DevBuf<uint32_t> res, F, next;
+  DevBuf<uint32_t> res, F, next, Fs, Fb, Fh;
   DevBuf<uint8_t> state;
-  DevBuf<unsigned> counters;  // [0] = |F| being built, [1] = |next|
+  DevBuf<unsigned> counters;  // [0] |F| being built, [1] |next|, [2] |Fs|, [3] |Fb|, [4] |Fh|
   res.alloc(n ? n : 1, s);
   F.alloc(n ? n : 1, s);
   next.alloc(n ? n : 1, s);
+  Fs.alloc(n ? n : 1, s);
+  Fb.alloc(n ? n : 1, s);
+  Fh.alloc(n ? n : 1, s);
   state.alloc(n ? n : 1, s);
-  counters.alloc(2, s);
+  counters.alloc(5, s);
   g.sub.alloc(n ? n : 1, s);
   g.dsnap.alloc(n ? n : 1, s);
   TC_CUDA(cudaMemcpyAsync(res.get(), g.deg.get(), sizeof(uint32_t) * n, cudaMemcpyDeviceToDevice, s));
@@ -210,12 +304,22 @@ void peel_paper(Graph &g) {
       TC_CUDA(cudaStreamSynchronize(s));
       unsigned nf = h_cnt[0];
       while (nf > 0) {
-        mark_kernel<<<grid_for(nf, 256), 256, 0, s>>>(F.get(), nf, state.get(), res.get(), g.sub.get(), g.dsnap.get(), r);
+        TC_CUDA(cudaMemsetAsync(counters.get() + 1, 0, 4 * sizeof(unsigned), s));
+        mark_kernel<<<grid_for(nf, 256), 256, 0, s>>>(F.get(), nf, state.get(), res.get(), g.deg.get(), g.sub.get(),
+                                                      g.dsnap.get(), r, Fs.get(), Fb.get(), Fh.get(),
+                                                      counters.get() + 2);
         TC_LAUNCH_CHECK();
-        TC_CUDA(cudaMemsetAsync(counters.get() + 1, 0, sizeof(unsigned), s));
-        expand_kernel<<<grid_for((uint64_t)nf * 32, 256), 256, 0, s>>>(F.get(), nf, soffs.get(), sadj.get(),
-                                                                       state.get(), res.get(), thr, next.get(),
-                                                                       counters.get() + 1);
+        // |Fs| and |Fb| stay on the device: both expands size their grids from nf
+        expand_flat_kernel<<<grid_for(((uint64_t)nf + 31) / 32 * 32, 256), 256, 0, s>>>(
+            Fs.get(), counters.get() + 2, soffs.get(), sadj.get(), state.get(), res.get(), thr, next.get(),
+            counters.get() + 1);
+        TC_LAUNCH_CHECK();
+        expand_kernel<<<grid_for((uint64_t)nf * 32, 256), 256, 0, s>>>(Fb.get(), counters.get() + 3, soffs.get(),
+                                                                       sadj.get(), state.get(), res.get(), thr,
+                                                                       next.get(), counters.get() + 1);
+        TC_LAUNCH_CHECK();
+        expand_huge_kernel<<<num_sms() * 4, 256, 0, s>>>(Fh.get(), counters.get() + 4, soffs.get(), sadj.get(),
+                                                         state.get(), res.get(), thr, next.get(), counters.get() + 1);
         TC_LAUNCH_CHECK();
         peel_kernel<<<grid_for(nf, 256), 256, 0, s>>>(F.get(), nf, state.get());
         TC_LAUNCH_CHECK();

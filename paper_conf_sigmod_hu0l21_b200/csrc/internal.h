@@ -93,5 +93,6 @@ extern int g_opt_profile;
 extern int g_opt_small_cap;
 extern int g_opt_l2_persist;
 extern int g_opt_bracket;
+extern int g_opt_split;  // orientation split CSR build (original labels)
 
 }  // namespace tc

@@ -193,6 +193,74 @@ __global__ __launch_bounds__(T_THREADS) void unique_kernel(const uint64_t *__res
   }
 }
 
+// ------------------------------------------------------------------ orientation split
+// Sorted undirected keys (a << bits) | b, a < b, are split by the orientation rule
+// u -> v iff (prim[u], u) < (prim[v], v): forward edges (a -> b) keep their key and their
+// order in F; reversed edges (b -> a) become (b << bits) | a in R, in input order (so each
+// source's group is ascending in a after a stable sort of R on the source bits).  One
+// look-back on the forward count per tile; the reversed position is (index - forward).
+__global__ __launch_bounds__(T_THREADS) void split_kernel(const uint64_t *__restrict__ in, uint64_t n, int bits,
+                                                          const uint64_t *__restrict__ prim, uint64_t *__restrict__ F,
+                                                          uint64_t *__restrict__ R, uint64_t *status,
+                                                          uint32_t *tile_ctr, uint64_t ntiles, uint64_t *d_nf) {
+  __shared__ uint32_t s_wcnt[T_WARPS];
+  __shared__ uint64_t s_base;
+  __shared__ uint32_t s_tile;
+  if (threadIdx.x == 0) s_tile = atomicAdd(tile_ctr, 1u);
+  __syncthreads();
+  const uint64_t tile = s_tile;
+  const unsigned w = warp_id(), l = lane_id();
+  const uint64_t wb = tile * T_TILE + (uint64_t)w * (32 * T_ITEMS);
+  const uint64_t mask = (1ull << bits) - 1;
+  uint64_t k[T_ITEMS];
+  unsigned fm[T_ITEMS];
+#pragma unroll
+  for (int i = 0; i < T_ITEMS; ++i) {
+    const uint64_t idx = wb + 32 * i + l;
+    k[i] = idx < n ? __ldcs(in + idx) : 0ull;
+  }
+  uint32_t wcnt = 0;
+#pragma unroll
+  for (int i = 0; i < T_ITEMS; ++i) {
+    const uint64_t idx = wb + 32 * i + l;
+    bool fwd = false;
+    if (idx < n) {
+      const uint32_t a = (uint32_t)(k[i] >> bits), b = (uint32_t)(k[i] & mask);
+      fwd = prim[a] <= prim[b];
+      if (!fwd) k[i] = ((uint64_t)b << bits) | a;
+    }
+    fm[i] = __ballot_sync(0xffffffffu, fwd);
+    wcnt += __popc(fm[i]);
+  }
+  if (l == 0) s_wcnt[w] = wcnt;
+  __syncthreads();
+  if (w == 0) {
+    const uint32_t c = l < T_WARPS ? s_wcnt[l] : 0u;
+    const uint32_t inc = warp_inclusive_scan(c);
+    const uint32_t total = __shfl_sync(0xffffffffu, inc, 31);
+    const uint64_t excl = warp_lookback(status, tile, total);
+    if (l < T_WARPS) s_wcnt[l] = inc - c;
+    if (l == 0) {
+      s_base = excl;
+      if (tile == ntiles - 1) *d_nf = excl + total;
+    }
+  }
+  __syncthreads();
+  uint64_t fpos = s_base + s_wcnt[w];  // forward edges before this warp's first key
+  const unsigned lt = (1u << l) - 1u;
+#pragma unroll
+  for (int i = 0; i < T_ITEMS; ++i) {
+    const uint64_t row = wb + 32 * i;  // keys before this row: row; forward among them: fpos
+    const uint64_t idx = row + l;
+    if (idx < n) {
+      const uint32_t fb = __popc(fm[i] & lt);
+      if (fm[i] >> l & 1u) F[fpos + fb] = k[i];
+      else R[(row - fpos) + (l - fb)] = k[i];
+    }
+    fpos += __popc(fm[i]);
+  }
+}
+
 // ------------------------------------------------------------------ radix sort
 // Up-front digit histograms for every pass; per-warp private smem counters.
 template <class Src>
@@ -440,6 +508,25 @@ void unique_sorted_u64(const uint64_t *in, uint64_t *out, uint64_t n, uint64_t *
   unique_kernel<<<(unsigned)ntiles, T_THREADS, 0, s>>>(in, out, n, scratch.get() + 1, (uint32_t *)scratch.get(),
                                                        ntiles, d_count, deg, bits, sentinel);
   TC_LAUNCH_CHECK();
+}
+
+uint64_t split_oriented(const uint64_t *edges, uint64_t m, int bits, const uint64_t *prim, uint64_t *F, uint64_t *R,
+                        cudaStream_t s) {
+  if (m == 0) return 0;
+  uint64_t ntiles = (m + T_TILE - 1) / T_TILE;
+  DevBuf<uint64_t> scratch;  // [tile counter | forward count][status ntiles]
+  scratch.alloc(ntiles + 2, s);
+  TC_CUDA(cudaMemsetAsync(scratch.get(), 0, scratch.bytes(), s));
+  {
+    ProfScope prof("split", s, 16.0 * m);
+    split_kernel<<<(unsigned)ntiles, T_THREADS, 0, s>>>(edges, m, bits, prim, F, R, scratch.get() + 2,
+                                                        (uint32_t *)scratch.get(), ntiles, scratch.get() + 1);
+    TC_LAUNCH_CHECK();
+  }
+  uint64_t nf = 0;
+  TC_CUDA(cudaMemcpyAsync(&nf, scratch.get() + 1, sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
+  TC_CUDA(cudaStreamSynchronize(s));
+  return nf;
 }
 
 template <class Src>

@@ -25,6 +25,12 @@ uint64_t *radix_sort_edges(const uint32_t *src, const uint32_t *dst, uint64_t M,
 void unique_sorted_u64(const uint64_t *in, uint64_t *out, uint64_t N, uint64_t *d_count, cudaStream_t s,
                        uint32_t *deg = nullptr, int bits = 0, uint64_t sentinel = 0);
 
+// Orientation split of sorted undirected keys (a << bits) | b (a < b): forward edges
+// (prim[a] <= prim[b]) keep key and order in F, reversed ones become (b << bits) | a in R in
+// input order.  Returns |F| (|R| = m - |F|).  Synchronises the stream.
+uint64_t split_oriented(const uint64_t *edges, uint64_t m, int bits, const uint64_t *prim, uint64_t *F, uint64_t *R,
+                        cudaStream_t s);
+
 // Block-wide exclusive scan helper (256 threads) used by several kernels.
 template <typename T>
 __device__ __forceinline__ T block256_exclusive_scan(T v, T *s_warp /*8 entries*/, T *total) {

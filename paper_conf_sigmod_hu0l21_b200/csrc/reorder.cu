@@ -14,6 +14,9 @@
 #include "prims.cuh"
 
 namespace tc {
+
+int g_opt_split = 1;
+
 namespace {
 
 __global__ void dorder_keys_kernel(const uint32_t *__restrict__ od, uint32_t n, uint32_t maxod, int bn,
@@ -69,8 +72,102 @@ __global__ void csr_ends_kernel(const uint64_t *__restrict__ keys, uint64_t m, i
   }
 }
 
+// ---- original labels: CSR from the orientation split (forward run F, sorted reversed run R)
+// lb[x] = first index of a key with source >= x in a source-sorted key array (x in [0, n]);
+// fused with the column fill of the same array: R entry i (source s) lands at
+// col[i + LF[s]] (R entries before it + F entries of smaller sources), F entry j at
+// col[j + LR[s + 1]] (all R entries of sources <= s precede it: they are smaller targets).
+template <bool IS_R>
+__global__ void lb_fill_kernel(const uint64_t *__restrict__ keys, uint64_t len, int bits, uint64_t *__restrict__ lb,
+                               const uint64_t *__restrict__ other_lb, uint32_t *__restrict__ col) {
+  const uint64_t mask = (1ull << bits) - 1;
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < len; i += (uint64_t)gridDim.x * blockDim.x) {
+    const uint64_t k = keys[i];
+    const uint64_t s = k >> bits;
+    const uint64_t x0 = i ? (keys[i - 1] >> bits) + 1 : 0;
+    for (uint64_t x = x0; x <= s; ++x) lb[x] = i;  // interior gaps are short
+    if (IS_R) col[i + other_lb[s]] = (uint32_t)(k & mask);
+  }
+}
+__global__ void lb_tail_kernel(const uint64_t *__restrict__ keys, uint64_t len, int bits, uint32_t n,
+                               uint64_t *__restrict__ lb) {
+  const uint64_t first = len ? (keys[len - 1] >> bits) + 1 : 0;
+  for (uint64_t x = first + (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; x <= n; x += (uint64_t)gridDim.x * blockDim.x)
+    lb[x] = len;
+}
+__global__ void fill_fwd_kernel(const uint64_t *__restrict__ F, uint64_t nf, int bits,
+                                const uint64_t *__restrict__ LR, uint32_t *__restrict__ col) {
+  const uint64_t mask = (1ull << bits) - 1;
+  for (uint64_t j = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; j < nf; j += (uint64_t)gridDim.x * blockDim.x) {
+    const uint64_t k = F[j];
+    col[j + LR[(k >> bits) + 1]] = (uint32_t)(k & mask);
+  }
+}
+__global__ void offs_sum_kernel(uint64_t *__restrict__ offs, const uint64_t *__restrict__ LR, uint32_t n) {
+  for (uint64_t x = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; x <= n; x += (uint64_t)gridDim.x * blockDim.x)
+    offs[x] += LR[x];
+}
+
 }  // namespace
 
+static void alloc_csr(Graph &g) {
+  cudaStream_t s = g.stream;
+  // [offs | col] in one allocation; col gets 32 words of tail padding (TMA bulk copies may
+  // over-read by < 16 B) and starts 16-B aligned
+  const uint64_t offs_words = ((uint64_t)g.n + 1 + 1) & ~1ull;
+  g.offs.release();
+  g.col.release();
+  g.csr_mem.alloc(offs_words + (g.m + 32 + 1) / 2, s);
+  g.offs = View<uint64_t>{g.csr_mem.get(), (size_t)g.n + 1};
+  g.col = View<uint32_t>{reinterpret_cast<uint32_t *>(g.csr_mem.get() + offs_words), (size_t)(g.m + 32)};
+  TC_CUDA(cudaMemsetAsync(g.col.get() + g.m, 0xff, 32 * sizeof(uint32_t), s));
+}
+
+// Original labels, any non-ID rule: the unique edge keys (a << b) | c, a < c, are already
+// sorted; the forward edges (a -> c) stay in that order, and only the reversed ones (c -> a)
+// need a STABLE sort on their source bits (b bits of |R| keys instead of all m keys).
+// N+(x) = R(x) ++ F(x): every reversed target is < x < every forward target, each run
+// ascending, so the lists come out sorted without a merge.
+static void build_csr_split(Graph &g) {
+  cudaStream_t s = g.stream;
+  const uint32_t n = g.n;
+  const uint64_t m = g.m;
+  const int b = g.bits;
+  DevBuf<uint64_t> F, R, tmp;
+  F.alloc(m, s);
+  R.alloc(m, s);
+  const uint64_t nf = split_oriented(g.edges.get(), m, b, g.prim.get(), F.get(), R.get(), s);
+  const uint64_t nr = m - nf;
+  uint64_t *Rs = R.get();
+  if (nr > 1) {
+    tmp.alloc(nr, s);
+    Rs = radix_sort_u64(R.get(), tmp.get(), nr, b, 2 * b, s);
+  }
+  alloc_csr(g);
+  DevBuf<uint64_t> LR;
+  LR.alloc((uint64_t)n + 1, s);
+  uint64_t *LF = g.offs.get();
+  ProfScope prof("csr_fill", s, 8.0 * m + 4.0 * m + 16.0 * ((double)n + 1));
+  if (nf) {
+    lb_fill_kernel<false><<<grid_for(nf, 256), 256, 0, s>>>(F.get(), nf, b, LF, nullptr, nullptr);
+    TC_LAUNCH_CHECK();
+  }
+  lb_tail_kernel<<<grid_for((uint64_t)n + 1, 256), 256, 0, s>>>(F.get(), nf, b, n, LF);
+  TC_LAUNCH_CHECK();
+  if (nr) {
+    lb_fill_kernel<true><<<grid_for(nr, 256), 256, 0, s>>>(Rs, nr, b, LR.get(), LF, g.col.get());
+    TC_LAUNCH_CHECK();
+  }
+  lb_tail_kernel<<<grid_for((uint64_t)n + 1, 256), 256, 0, s>>>(Rs, nr, b, n, LR.get());
+  TC_LAUNCH_CHECK();
+  if (nf) {
+    fill_fwd_kernel<<<grid_for(nf, 256), 256, 0, s>>>(F.get(), nf, b, LR.get(), g.col.get());
+    TC_LAUNCH_CHECK();
+  }
+  offs_sum_kernel<<<grid_for((uint64_t)n + 1, 256), 256, 0, s>>>(LF, LR.get(), n);
+  TC_LAUNCH_CHECK();
+  g.csr_ready = true;
+}
 
 void build_oriented_csr(Graph &g) {
   cudaStream_t s = g.stream;
@@ -78,6 +175,10 @@ void build_oriented_csr(Graph &g) {
   const uint64_t m = g.m;
   const int b = g.bits;
   const bool ident = g.identity_perm;
+  if (ident && g.direct_rule != TC_DIRECT_ID && m && g_opt_split) {
+    build_csr_split(g);
+    return;
+  }
   DevBuf<uint64_t> keys, tmp;
   keys.alloc(m ? m : 1, s);
   if (m) {
@@ -102,15 +203,7 @@ void build_oriented_csr(Graph &g) {
     tmp.alloc(m ? m : 1, s);
     sorted = radix_sort_u64(keys.get(), tmp.get(), m, 0, 2 * b, s);
   }
-  // [offs | col] in one allocation; col gets 32 words of tail padding (TMA bulk copies may
-  // over-read by < 16 B) and starts 16-B aligned
-  const uint64_t offs_words = ((uint64_t)n + 1 + 1) & ~1ull;
-  g.offs.release();
-  g.col.release();
-  g.csr_mem.alloc(offs_words + (m + 32 + 1) / 2, s);
-  g.offs = View<uint64_t>{g.csr_mem.get(), (size_t)n + 1};
-  g.col = View<uint32_t>{reinterpret_cast<uint32_t *>(g.csr_mem.get() + offs_words), (size_t)(m + 32)};
-  TC_CUDA(cudaMemsetAsync(g.col.get() + m, 0xff, 32 * sizeof(uint32_t), s));
+  alloc_csr(g);
   if (m) {
     ProfScope prof("extract_csr", s, 12.0 * m);
     extract_csr_kernel<<<grid_for(m, 256), 256, 0, s>>>(sorted, m, b, n, g.col.get(), g.offs.get());
