@@ -66,21 +66,6 @@ __device__ __forceinline__ bool bsearch_list(const uint32_t *s, uint32_t L, uint
   return *p == w;
 }
 
-// Fixed-depth search over a list padded with +inf (0xffffffff, never a vertex id) to 2^S
-// entries: S unrolled steps of one shared load + compare + select each ("binary lifting").
-// Precondition: s[0] <= w (the caller's range filter).
-// Returns the position p of the last element <= w (hit iff tc_smem[p] == w).
-template <int S>
-__device__ __forceinline__ uint32_t bsearch_pow2(uint32_t sbase, uint32_t w) {
-  uint32_t p = sbase;
-#pragma unroll
-  for (int k = S - 1; k >= 0; --k) {
-    uint32_t q = p + (1u << k);
-    p = (tc_smem[q] <= w) ? q : p;
-  }
-  return p;
-}
-
 __device__ __forceinline__ int ceil_log2(uint32_t L) { return L <= 1 ? 0 : 32 - __clz(L - 1); }
 
 // words of dynamic shared memory per warp in the warp-item kernels
@@ -100,12 +85,39 @@ struct GlobalSearch {  // N+(u) in global memory (lists longer than a warp slice
     return bsearch_list(list, L, w);
   }
 };
+// Shared-memory loads through 32-bit shared-window byte addresses computed once per
+// item (the generic tc_smem[] form made the compiler rebuild the window base from
+// SR_CgaCtaId on every probe: 4 uniform instructions per wedge).
+__device__ __forceinline__ uint32_t smem_addr(uint32_t word) {
+  return (uint32_t)__cvta_generic_to_shared(tc_smem) + 4u * word;
+}
+__device__ __forceinline__ uint32_t lds32(uint32_t a) {
+  uint32_t v;
+  asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(a) : "memory");
+  return v;
+}
+__device__ __forceinline__ uint32_t lds16(uint32_t a) {
+  unsigned short v;
+  asm volatile("ld.shared.u16 %0, [%1];" : "=h"(v) : "r"(a) : "memory");
+  return v;
+}
+
+// All searches are branch-free and valid for ANY vertex id w (no [lo, hi] pre-filter is
+// needed): a w outside the list's range ends on an element != w (ids are < 2^32 - 1, so
+// never equal to the +inf padding).
 template <int S>
 struct Pow2Search {  // full fixed-depth binary search over the +inf-padded slice
-  uint32_t sbase;
+  uint32_t sa;       // byte address of slice[0]
+  uint32_t sbase;    // word index of slice[0] (PV positions)
   __device__ __forceinline__ bool operator()(uint32_t w, uint32_t &pos) const {
-    pos = bsearch_pow2<S>(sbase, w);
-    return tc_smem[pos] == w;
+    uint32_t p = sa;
+#pragma unroll
+    for (int k = S - 1; k >= 0; --k) {
+      const uint32_t q = p + (4u << k);
+      p = (lds32(q) <= w) ? q : p;
+    }
+    pos = sbase + ((p - sa) >> 2);
+    return lds32(p) == w;
   }
 };
 // Bracketed binary search: a per-item table maps the value bucket (w - lo) >> sh to the
@@ -113,18 +125,21 @@ struct Pow2Search {  // full fixed-depth binary search over the +inf-padded slic
 // (S2 = ceil(log2 max bucket occupancy) steps instead of ceil(log2 d~(u))).  Elements
 // past the bucket are larger than w (buckets are monotone), and the slice carries +inf
 // padding past its end, so no bounds checks are needed.
+// A w outside [lo, hi] maps to bucket B (clamped), whose entry is L: the probes then read
+// the +inf padding (2^S2 - 1 < 64 entries past L) and end on an element != w.
 template <int S2>
 struct TabSearch {
-  uint32_t sbase, tbase, lo, sh;
+  uint32_t sa, ta, lo, sh, B, sbase;  // slice / table byte addresses, table size, PV base
   __device__ __forceinline__ bool operator()(uint32_t w, uint32_t &pos) const {
-    uint32_t p = sbase + reinterpret_cast<const uint16_t *>(tc_smem + tbase)[(w - lo) >> sh];
+    const uint32_t b = min((w - lo) >> sh, B);
+    uint32_t p = sa + 4u * lds16(ta + 2u * b);
 #pragma unroll
     for (int k = S2 - 1; k >= 0; --k) {
-      uint32_t q = p + (1u << k);
-      p = (tc_smem[q] <= w) ? q : p;
+      const uint32_t q = p + (4u << k);
+      p = (lds32(q) <= w) ? q : p;
     }
-    pos = p;
-    return tc_smem[p] == w;
+    pos = sbase + ((p - sa) >> 2);
+    return lds32(p) == w;
   }
 };
 
@@ -140,46 +155,43 @@ __device__ __forceinline__ uint32_t wedge_loop(const uint32_t *__restrict__ col,
                                                uint32_t cbase, uint32_t lo, uint32_t hi, uint32_t total,
                                                WarpScratch &ws, unsigned long long *tv) {
   uint32_t cnt = 0;
-  uint32_t o = 0, o_beg = 0, o_end = ws.pre[0];
-  uint64_t o_vb = ws.vb[0];
+  uint32_t o = 0, o_end = ws.pre[0];
+  const uint32_t *ob = col + ws.vb[0];  // element j of the current owner list is ob[j]
   // UNR wedges per lane in flight: their loads are issued back to back before any search
-  // (memory-level parallelism for the gather; the owner walk stays incremental).
+  // (memory-level parallelism for the gather; the owner walk stays incremental).  The
+  // tail is branch-free: indices past `total` are clamped to the last wedge (a valid
+  // address) and their hits masked (a clamped w must not count twice; +inf would match
+  // the padding).
   constexpr int UNR = 4;
+  const uint32_t last = total - 1;
   for (uint32_t j0 = lane_id(); j0 < total; j0 += 32 * UNR) {
     uint32_t w[UNR], ow[UNR];
 #pragma unroll
     for (int k = 0; k < UNR; ++k) {
-      const uint32_t j = j0 + 32 * k;
-      w[k] = 0xffffffffu;  // > hi: filtered out
-      ow[k] = o;
-      if (j < total) {
-        if (o_end <= j) {
-          do {
-            ++o;
-            o_beg = o_end;
-            o_end = ws.pre[o];
-          } while (o_end <= j);
-          o_vb = ws.vb[o];
-        }
-        ow[k] = o;
-        w[k] = ldg_u32(col + o_vb + (j - o_beg));
+      const uint32_t j = min(j0 + 32 * k, last);
+      while (o_end <= j) {
+        const uint32_t o_beg = o_end;
+        ++o;
+        o_end = ws.pre[o];
+        ob = col + ws.vb[o] - o_beg;
       }
+      ow[k] = o;
+      w[k] = ldg_u32(ob + j);
     }
 #pragma unroll
     for (int k = 0; k < UNR; ++k) {
-      if (w[k] >= lo && w[k] <= hi) {
-        uint32_t pos;
-        if (search(w[k], pos)) {
-          ++cnt;
-          if (PV) {
-            atomicAdd(&ws.vcnt[ow[k]], 1u);
-            if (cbase != 0xffffffffu) atomicAdd(&tc_smem[cbase + (pos - sbase)], 1u);
-            else atomicAdd(&tv[w[k]], 1ull);
-          }
-        }
+      uint32_t pos;
+      const bool hit = search(w[k], pos) && j0 + 32 * k <= last;
+      cnt += hit ? 1u : 0u;
+      if (PV && hit) {
+        atomicAdd(&ws.vcnt[ow[k]], 1u);
+        if (cbase != 0xffffffffu) atomicAdd(&tc_smem[cbase + (pos - sbase)], 1u);
+        else atomicAdd(&tv[w[k]], 1ull);
       }
     }
   }
+  (void)lo;
+  (void)hi;
   return cnt;
 }
 
@@ -246,14 +258,17 @@ __device__ __forceinline__ uint32_t warp_chunk(const uint64_t *__restrict__ offs
     if (S2 <= 6) {
       switch (S2) {
 #define TC_TAB(k) \
-  case k: cnt = wedge_loop<PV>(col, TabSearch<k>{sbase, tbase, lo, sh}, sbase, cbase, lo, hi, total, ws, tv); break;
+  case k:                                                                                                     \
+    cnt = wedge_loop<PV>(col, TabSearch<k>{smem_addr(sbase), smem_addr(tbase), lo, sh, ((hi - lo) >> sh) + 1, sbase}, \
+                         sbase, cbase, lo, hi, total, ws, tv);                                                \
+    break;
         TC_TAB(0) TC_TAB(1) TC_TAB(2) TC_TAB(3) TC_TAB(4) TC_TAB(5) TC_TAB(6)
 #undef TC_TAB
       }
     } else {
       switch (S) {
 #define TC_CASE(k) \
-  case k: cnt = wedge_loop<PV>(col, Pow2Search<k>{sbase}, sbase, cbase, lo, hi, total, ws, tv); break;
+  case k: cnt = wedge_loop<PV>(col, Pow2Search<k>{smem_addr(sbase), sbase}, sbase, cbase, lo, hi, total, ws, tv); break;
         TC_CASE(1) TC_CASE(2) TC_CASE(3) TC_CASE(4) TC_CASE(5) TC_CASE(6) TC_CASE(7)
         TC_CASE(8) TC_CASE(9) TC_CASE(10) TC_CASE(11) TC_CASE(12) TC_CASE(13) TC_CASE(14)
 #undef TC_CASE
@@ -403,7 +418,7 @@ __global__ __launch_bounds__(256) void items_scatter_kernel(const uint64_t *__re
 // --------------------------------------------------------------- count kernels (a9)
 // Warp items; items [0, nheavy) are fetched one at a time, the rest CHUNK at a time.
 template <bool PV>
-__global__ __launch_bounds__(CT_THREADS) void count_small_kernel(const uint64_t *__restrict__ offs,
+__global__ __launch_bounds__(CT_THREADS, 6) void count_small_kernel(const uint64_t *__restrict__ offs,
                                                                  const uint32_t *__restrict__ col,
                                                                  const uint64_t *__restrict__ items, uint64_t nitems,
                                                                  uint64_t nheavy, unsigned long long *ctr, uint32_t cap,
@@ -466,7 +481,7 @@ __device__ __forceinline__ void mbar_wait(uint64_t *bar, unsigned phase) {
 // CTA items (u, c0) of heavy sources: v's N+(u)[c0 .. c0+LV) over 16 warps; N+(u) staged
 // piece by piece with a TMA bulk copy (cp.async.bulk + mbarrier complete_tx).
 template <bool PV>
-__global__ __launch_bounds__(LG_THREADS) void count_large_kernel(const uint64_t *__restrict__ offs,
+__global__ __launch_bounds__(LG_THREADS, 5) void count_large_kernel(const uint64_t *__restrict__ offs,
                                                                  const uint32_t *__restrict__ col,
                                                                  const uint64_t *__restrict__ items, uint64_t nitems,
                                                                  unsigned long long *ctr, unsigned long long *T,
