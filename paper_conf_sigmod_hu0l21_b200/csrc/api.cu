@@ -183,6 +183,7 @@ tc_status tc_set_option(const char *key, int64_t value) {
     else if (k == "l2_persist") g_opt_l2_persist = value ? 1 : 0;
     else if (k == "trim_memory") dev_trim();
     else if (k == "bracket") g_opt_bracket = value ? 1 : 0;
+    else if (k == "peel_coop") g_opt_peel_coop = value ? 1 : 0;
     else if (k == "split") g_opt_split = value ? 1 : 0;
     else if (k == "small_cap") {
       TC_REQUIRE(value >= 32 && value <= 2048 && (value & (value - 1)) == 0, ST_INVALID,

@@ -18,11 +18,14 @@
 // doubles it (line 19).  The sequential oracle (oracle/tc_oracle.c) and this BSP form yield
 // the same orientation because decrements commute and dsnap is taken after the previous
 // subround completes.
+#include <cooperative_groups.h>
+
 #include "internal.h"
 #include "prims.cuh"
 
 namespace tc {
 
+int g_opt_peel_coop = 1;  // whole A-direction peel in one cooperative launch
 
 namespace {
 
@@ -79,8 +82,9 @@ __global__ void frontier_init_kernel(const uint8_t *__restrict__ state, const ui
 // Marks the frontier (snapshot at formation) and splits it by degree for the three expand
 // kernels: d(v) <= 32 -> Fs (flattened, 32 vertices per warp), 32 < d(v) <= HUGE_DEG -> Fb
 // (warp per vertex), d(v) > HUGE_DEG -> Fh (the whole grid per vertex: a hub never
-// serialises on one warp).  Vertices with d(v) = 0 have nothing to expand.
-constexpr uint32_t HUGE_DEG = 4096;
+// serialises on one warp; hubs are cut into chunks of HUB_CHUNK edges spread over all warps).
+// Vertices with d(v) = 0 have nothing to expand.
+constexpr uint32_t HUGE_DEG = 1024;
 __global__ void mark_kernel(const uint32_t *__restrict__ F, unsigned nf, uint8_t *state,
                             const uint32_t *__restrict__ res, const uint32_t *__restrict__ deg, uint32_t *sub,
                             uint32_t *dsnap, uint32_t r, uint32_t *Fs, uint32_t *Fb, uint32_t *Fh,
@@ -176,28 +180,235 @@ __global__ void expand_kernel(const uint32_t *__restrict__ F, const unsigned *__
   }
 }
 
-// Frontier hubs (d(v) > HUGE_DEG), one after another, each spread over every thread of
-// the grid; the appends stay warp-aggregated.
-__global__ void expand_huge_kernel(const uint32_t *__restrict__ F, const unsigned *__restrict__ nfp,
-                                   const uint64_t *__restrict__ soffs, const uint32_t *__restrict__ sadj,
-                                   const uint8_t *__restrict__ state, uint32_t *res, uint64_t thr, uint32_t *next,
-                                   unsigned *nnext) {
-  const unsigned nf = *nfp;
-  const uint64_t nthreads = (uint64_t)gridDim.x * blockDim.x;
-  const uint64_t tid0 = (uint64_t)blockIdx.x * blockDim.x + (threadIdx.x & ~31u);
-  for (unsigned i = 0; i < nf; ++i) {
+// Frontier hubs (d(v) > HUGE_DEG): cut into chunks of HUB_CHUNK edges, one warp per chunk
+// over the whole grid.  Every CTA builds the chunk prefix of the (few) hubs in shared
+// memory and binary-searches it per chunk; with more than HUB_MAX hubs the hubs are taken
+// one after another, each spread over every thread of the grid.  Called by whole CTAs.
+constexpr uint32_t HUB_CHUNK = 1024, HUB_MAX = 8192;
+__device__ __forceinline__ void expand_hubs(const uint32_t *__restrict__ F, unsigned nh,
+                                            const uint64_t *__restrict__ soffs, const uint32_t *__restrict__ sadj,
+                                            const uint8_t *__restrict__ state, uint32_t *res, uint64_t thr,
+                                            uint32_t *next, unsigned *nnext, uint32_t *s_pre) {
+  const unsigned lane = lane_id();
+  const uint64_t gthreads = (uint64_t)gridDim.x * blockDim.x;
+  const uint64_t gtid0 = (uint64_t)blockIdx.x * blockDim.x + (threadIdx.x & ~31u);
+  if (nh == 0) return;
+  if (nh > HUB_MAX) {
+    for (unsigned i = 0; i < nh; ++i) {
+      const uint32_t v = F[i];
+      const uint64_t a = soffs[v], e = soffs[v + 1];
+      for (uint64_t p0 = a + gtid0; p0 < e; p0 += gthreads) {
+        const uint64_t p = p0 + lane;
+        bool cross = false;
+        uint32_t nbr = 0;
+        if (p < e) {
+          nbr = sadj[p];
+          cross = expand_one(nbr, state, res, thr);
+        }
+        warp_append(cross, nbr, next, nnext);
+      }
+    }
+    return;
+  }
+  // inclusive prefix of chunk counts: thread t sums a contiguous run, block scan, write back
+  __shared__ uint32_t s_tot[32];
+  const unsigned per = (nh + blockDim.x - 1) / blockDim.x;
+  const unsigned b0 = threadIdx.x * per, b1 = min(nh, b0 + per);
+  uint32_t run = 0;
+  for (unsigned i = b0; i < b1; ++i) {
     const uint32_t v = F[i];
-    const uint64_t a = soffs[v], e = soffs[v + 1];
-    for (uint64_t p0 = a + tid0; p0 < e; p0 += nthreads) {
-      const uint64_t p = p0 + lane_id();
+    run += (uint32_t)((soffs[v + 1] - soffs[v] + HUB_CHUNK - 1) / HUB_CHUNK);
+    s_pre[i] = run;
+  }
+  const uint32_t inc = warp_inclusive_scan(run);
+  if (lane == 31) s_tot[warp_id()] = inc;
+  __syncthreads();
+  if (warp_id() == 0) {
+    const unsigned nw = blockDim.x / 32;
+    const uint32_t x = lane < nw ? s_tot[lane] : 0u;
+    const uint32_t xi = warp_inclusive_scan(x);
+    if (lane < nw) s_tot[lane] = xi - x;
+  }
+  __syncthreads();
+  const uint32_t add = inc - run + s_tot[warp_id()];
+  for (unsigned i = b0; i < b1; ++i) s_pre[i] += add;
+  __syncthreads();
+  const uint32_t total = s_pre[nh - 1];
+  const unsigned nwarps = (unsigned)(gthreads >> 5);
+  for (uint32_t c = (uint32_t)(gtid0 >> 5); c < total; c += nwarps) {
+    unsigned lo = 0, hi = nh - 1;  // first i with s_pre[i] > c
+    while (lo < hi) {
+      const unsigned mid = (lo + hi) >> 1;
+      if (s_pre[mid] > c) hi = mid;
+      else lo = mid + 1;
+    }
+    const uint32_t ci = c - (lo ? s_pre[lo - 1] : 0u);
+    const uint32_t v = F[lo];
+    const uint64_t e = soffs[v + 1];
+    const uint64_t a = soffs[v] + (uint64_t)ci * HUB_CHUNK;
+    const uint64_t ce = min(e, a + HUB_CHUNK);
+    for (uint64_t p0 = a; p0 < ce; p0 += 32) {
+      const uint64_t p = p0 + lane;
       bool cross = false;
       uint32_t nbr = 0;
-      if (p < e) {
+      if (p < ce) {
         nbr = sadj[p];
         cross = expand_one(nbr, state, res, thr);
       }
       warp_append(cross, nbr, next, nnext);
     }
+  }
+  __syncthreads();  // s_pre reusable
+}
+
+__global__ __launch_bounds__(256) void expand_huge_kernel(const uint32_t *__restrict__ F,
+                                                          const unsigned *__restrict__ nfp,
+                                                          const uint64_t *__restrict__ soffs,
+                                                          const uint32_t *__restrict__ sadj,
+                                                          const uint8_t *__restrict__ state, uint32_t *res,
+                                                          uint64_t thr, uint32_t *next, unsigned *nnext) {
+  __shared__ uint32_t s_pre[HUB_MAX];
+  expand_hubs(F, *nfp, soffs, sadj, state, res, thr, next, nnext, s_pre);
+}
+
+// ---------------------------------------------------------------- whole peel, one launch
+// The same BSP subrounds as the kernels above, run by ONE cooperative grid (every CTA
+// resident) with grid-wide barriers between the phases: no host round trip per subround
+// (the multi-launch loop paid a launch + a D2H copy + a stream sync per subround, ~30 per
+// R-MAT s22 run).  Frontier counters are read by every thread after a barrier and reset by
+// thread 0 one phase before their next use (double-buffered where a read and the next
+// reset would otherwise race).
+struct PeelArgs {
+  const uint64_t *soffs;
+  const uint32_t *sadj;
+  const uint32_t *deg;
+  uint32_t *res, *sub, *dsnap;
+  uint8_t *state;
+  uint32_t *F, *next, *Fs, *Fb, *Fh;
+  unsigned *ctr;      // [0,1] init-frontier counts (per level parity), [2,3] next counts, [4..6] split counts
+  uint32_t *out;      // [0] levels, [1] subrounds, [2] error
+  uint32_t n;
+  uint64_t m;
+};
+
+__global__ __launch_bounds__(256) void peel_coop_kernel(PeelArgs A) {
+  namespace cg = cooperative_groups;
+  __shared__ uint32_t s_pre[HUB_MAX];
+  cg::grid_group grid = cg::this_grid();
+  const uint64_t gtid = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  const uint64_t gthreads = (uint64_t)gridDim.x * blockDim.x;
+  const unsigned gwarp = (unsigned)(gtid >> 5), nwarps = (unsigned)(gthreads >> 5);
+  const unsigned lane = lane_id();
+  const uint32_t n = A.n;
+  uint64_t peeled = 0;
+  uint32_t level = 0, r = 0;
+  uint32_t *F = A.F, *next = A.next;
+  while (peeled < n) {
+    if (level >= 200) {  // cannot happen (thr reaches max degree after <= 64 levels)
+      if (gtid == 0) A.out[2] = 1;
+      break;
+    }
+    const unsigned __int128 t128 = ((unsigned __int128)A.m << level) / n;
+    const uint64_t thr = t128 > 0xFFFFFFFFull ? 0xFFFFFFFFull : (uint64_t)t128;
+    unsigned *cinit = A.ctr + (level & 1);
+    // frontier formation (Algorithm 1 line 4-6)
+    for (uint64_t base = gtid & ~31ull; base < n; base += gthreads) {
+      const uint64_t v = base + lane;
+      const bool want = v < n && A.state[v] == V_UNPEELED && (uint64_t)A.res[v] <= thr;
+      warp_append(want, (uint32_t)v, F, cinit);
+    }
+    grid.sync();
+    unsigned nf = *cinit;
+    if (gtid == 0) A.ctr[(level + 1) & 1] = 0;  // next level's init counter
+    while (nf > 0) {
+      unsigned *cnext = A.ctr + 2 + (r & 1);
+      // mark + split by degree
+      for (uint64_t base = gtid & ~31ull; base < nf; base += gthreads) {
+        const uint64_t i = base + lane;
+        uint32_t v = 0, d = 0;
+        if (i < nf) {
+          v = F[i];
+          A.state[v] = V_FRONTIER;
+          A.sub[v] = r;
+          A.dsnap[v] = A.res[v];
+          d = A.deg[v];
+        }
+        warp_append(i < nf && d != 0 && d <= 32, v, A.Fs, A.ctr + 4);
+        warp_append(i < nf && d > 32 && d <= HUGE_DEG, v, A.Fb, A.ctr + 5);
+        warp_append(i < nf && d > HUGE_DEG, v, A.Fh, A.ctr + 6);
+      }
+      grid.sync();
+      const unsigned ns = A.ctr[4], nb = A.ctr[5], nh = A.ctr[6];
+      // expand: d <= 32 flattened, 32 vertices per warp
+      for (unsigned g0 = gwarp * 32; g0 < ns; g0 += nwarps * 32) {
+        uint64_t a = 0;
+        uint32_t d = 0;
+        if (g0 + lane < ns) {
+          const uint32_t v = A.Fs[g0 + lane];
+          a = A.soffs[v];
+          d = (uint32_t)(A.soffs[v + 1] - a);
+        }
+        const uint32_t inc = warp_inclusive_scan(d);
+        const uint32_t total = __shfl_sync(0xffffffffu, inc, 31);
+        for (uint32_t j0 = 0; j0 < total; j0 += 32) {
+          const uint32_t j = j0 + lane;
+          uint32_t o = 0;
+#pragma unroll
+          for (int k = 4; k >= 0; --k) {
+            const uint32_t q = o + (1u << k);
+            const uint32_t pq = __shfl_sync(0xffffffffu, inc, (q - 1) & 31);
+            if (q <= 32 && pq <= j) o = q;
+          }
+          const uint32_t oo = o & 31;
+          const uint64_t ao = __shfl_sync(0xffffffffu, a, oo);
+          const uint32_t eo = __shfl_sync(0xffffffffu, inc, oo) - __shfl_sync(0xffffffffu, d, oo);
+          bool cross = false;
+          uint32_t nbr = 0;
+          if (j < total) {
+            nbr = A.sadj[ao + (j - eo)];
+            cross = expand_one(nbr, A.state, A.res, thr);
+          }
+          warp_append(cross, nbr, next, cnext);
+        }
+      }
+      // 32 < d <= HUGE_DEG: warp per vertex
+      for (unsigned i = gwarp; i < nb; i += nwarps) {
+        const uint32_t v = A.Fb[i];
+        const uint64_t a = A.soffs[v], e = A.soffs[v + 1];
+        for (uint64_t p0 = a; p0 < e; p0 += 32) {
+          const uint64_t p = p0 + lane;
+          bool cross = false;
+          uint32_t nbr = 0;
+          if (p < e) {
+            nbr = A.sadj[p];
+            cross = expand_one(nbr, A.state, A.res, thr);
+          }
+          warp_append(cross, nbr, next, cnext);
+        }
+      }
+      // hubs: chunks of HUB_CHUNK edges over every warp of the grid
+      expand_hubs(A.Fh, nh, A.soffs, A.sadj, A.state, A.res, thr, next, cnext, s_pre);
+      grid.sync();
+      // peel the frontier (Algorithm 1 line 17-18); reset the split counters and the
+      // next-frontier counter of the following subround
+      for (uint64_t i = gtid; i < nf; i += gthreads) A.state[F[i]] = V_PEELED;
+      if (gtid == 0) {
+        A.ctr[4] = A.ctr[5] = A.ctr[6] = 0;
+        A.ctr[2 + ((r + 1) & 1)] = 0;
+      }
+      grid.sync();
+      peeled += nf;
+      nf = *cnext;
+      ++r;
+      uint32_t *t = F;
+      F = next;
+      next = t;
+    }
+    ++level;
+  }
+  if (gtid == 0) {
+    A.out[0] = level;
+    A.out[1] = r;
   }
 }
 
@@ -281,11 +492,41 @@ void peel_paper(Graph &g) {
   Fb.alloc(n ? n : 1, s);
   Fh.alloc(n ? n : 1, s);
   state.alloc(n ? n : 1, s);
-  counters.alloc(5, s);
+  counters.alloc(8, s);
   g.sub.alloc(n ? n : 1, s);
   g.dsnap.alloc(n ? n : 1, s);
   TC_CUDA(cudaMemcpyAsync(res.get(), g.deg.get(), sizeof(uint32_t) * n, cudaMemcpyDeviceToDevice, s));
   TC_CUDA(cudaMemsetAsync(state.get(), 0, n, s));
+  if (g_opt_peel_coop) {
+    int dev = 0, coop = 0, occ = 0;
+    TC_CUDA(cudaGetDevice(&dev));
+    TC_CUDA(cudaDeviceGetAttribute(&coop, cudaDevAttrCooperativeLaunch, dev));
+    TC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, peel_coop_kernel, 256, 0));
+    if (coop && occ > 0) {
+      DevBuf<uint32_t> out;
+      out.alloc(3, s);
+      TC_CUDA(cudaMemsetAsync(out.get(), 0, 3 * sizeof(uint32_t), s));
+      TC_CUDA(cudaMemsetAsync(counters.get(), 0, counters.bytes(), s));
+      PeelArgs A{soffs.get(), sadj.get(), g.deg.get(), res.get(), g.sub.get(), g.dsnap.get(), state.get(),
+                 F.get(), next.get(), Fs.get(), Fb.get(), Fh.get(), counters.get(), out.get(), n, m};
+      void *args[] = {&A};
+      {
+        ProfScope prof("peel", s, 0.0);
+        TC_CUDA(cudaLaunchCooperativeKernel((const void *)peel_coop_kernel, dim3(num_sms() * occ), dim3(256), args, 0,
+                                            s));
+        TC_LAUNCH_CHECK();
+      }
+      uint32_t h_out[3] = {0, 0, 0};
+      TC_CUDA(cudaMemcpyAsync(h_out, out.get(), sizeof(h_out), cudaMemcpyDeviceToHost, s));
+      TC_CUDA(cudaStreamSynchronize(s));
+      TC_REQUIRE(h_out[2] == 0, ST_CUDA, "A-direction did not terminate");
+      g.levels = h_out[0];
+      g.subrounds = h_out[1];
+      prim_paper_kernel<<<grid_for(n, 256), 256, 0, s>>>(g.sub.get(), g.dsnap.get(), g.prim.get(), n);
+      TC_LAUNCH_CHECK();
+      return;
+    }
+  }
   // pinned frontier counters, allocated once per host thread (cudaMallocHost is slow)
   static thread_local unsigned *h_cnt = nullptr;
   if (!h_cnt) TC_CUDA(cudaMallocHost(&h_cnt, 2 * sizeof(unsigned)));
