@@ -125,6 +125,16 @@ tc_status tc_set_schedule(tc_graph *g, tc_schedule s);
  * receive t(v) indexed by ORIGINAL vertex id (Q23). */
 tc_status tc_count(tc_graph *g, uint64_t *triangles, uint64_t *per_vertex);
 
+/* Per-edge triangle counts ("support", the input of k-truss; P:15 and
+ * P:61 name TC's uses).  per_edge[e] = number of triangles containing the e-th edge of the
+ * simple undirected graph in canonical order — the order of tc_export_graph's `edges`
+ * (keys (min << 32) | max over the caller's vertex ids, ascending) — so it does not depend
+ * on the directing or ordering rule.  m entries, host or device memory (caller-owned);
+ * *triangles receives T.  Same kernels as tc_count, with three aggregated increments per
+ * triangle (edges (u,v), (u,w), (v,w) of u -> v -> w).  Requires tc_direct; errors as
+ * tc_count (TC_ERR_INVALID when per_edge is NULL and m > 0). */
+tc_status tc_count_edges(tc_graph *g, uint64_t *triangles, uint64_t *per_edge);
+
 /* Count only triangles whose source vertex (the lowest in the orientation) has a
  * new label in [u_begin, u_end); per_vertex (optional, n entries) receives this
  * slice's contributions (original ids).  The sum over a partition of [0,n) is T. */

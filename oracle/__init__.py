@@ -8,7 +8,7 @@ pins).  It shares no code with ``paper_conf_sigmod_hu0l21_b200`` and never
 imports it.
 
 Parity status:
-  * count T, per-vertex t(v), simple graph, ID/degree directing, D-order: pinned
+  * count T, per-vertex t(v), per-edge support, simple graph, ID/degree directing, D-order: pinned
     (closed forms, brute force, invariants).
   * A-direction (Alg.1) and A-order (Alg.2): "parity unpinned" against the
     authors' code (no worked example survives in PAPER.md); pinned only by hand
@@ -70,6 +70,7 @@ def lib():
         L.orc_count_forward.restype = u64
         L.orc_local_triangles.argtypes = [p, p, u64, p, u32, u32, p]
         L.orc_local_triangles.restype = i32
+        L.orc_edge_support.argtypes = [p, u64, p, p, p]
         _LIB = L
     return _LIB
 
@@ -189,6 +190,17 @@ def local_triangles(src, dst, vertices, max_deg=4096):
     return out[: len(vs)]
 
 
+def edge_support(edges, n, subset=None):
+    """Per-edge triangle counts |N(a) ∩ N(b)| in canonical edge order; `subset` (keys of
+    edges of the graph) restricts the output to those edges (sampled full-size parity)."""
+    offs, adj = sym_csr(edges, n)
+    q = edges if subset is None else np.ascontiguousarray(subset, dtype=np.uint64)
+    out = np.zeros(max(len(q), 1), dtype=np.uint64)
+    adj = adj if len(adj) else np.zeros(1, dtype=np.uint32)
+    lib().orc_edge_support(_p(q), len(q), _p(offs), _p(adj), _p(out))
+    return out[:len(q)]
+
+
 def cost_eq1(n, m, od):
     lo = np.zeros(1, dtype=np.uint64)
     hi = np.zeros(1, dtype=np.uint64)
@@ -228,7 +240,7 @@ def range_buckets(od, perm, k):
 
 def run(src, dst, n, direct_rule="degree", reorder_rule="none", per_vertex=False,
         k=DEFAULT_K, lam=DEFAULT_LAMBDA, alpha=DEFAULT_ALPHA, beta=DEFAULT_BETA, bw=None,
-        order=0):
+        order=0, per_edge=False):
     """The whole path on the CPU: O1 -> O2 -> O3 -> oriented CSR -> O4.
 
     Returns a dict: m, edges, deg, dir, od, perm, bucket_off, offs, col, T,
@@ -250,4 +262,6 @@ def run(src, dst, n, direct_rule="degree", reorder_rule="none", per_vertex=False
     else:
         T = count_forward(offs, col)
     res["T"] = T
+    if per_edge:
+        res["te"] = edge_support(edges, n)
     return res

@@ -34,6 +34,13 @@
  *                        friendship/book graphs, cycles, cocktail party),
  *                        brute-force trace(A^3)/6, node-iterator, Σt = 3T,
  *                        invariance over all 3x3 rules and relabelings.
+ *   orc_edge_support     per-edge triangle counts (support):
+ *                        support(a,b) = |N(a) ∩ N(b)| for every edge of the simple graph,
+ *                        by two-pointer merge of the two ascending SYMMETRIC lists (the
+ *                        plain definition: a triangle through {a,b} is a common
+ *                        neighbour).  pinned: Σ support = 3T, closed forms (K_n: n-2;
+ *                        wheel: spokes 2, rim 1; book: spine k, pages 1; friendship: 1;
+ *                        K_{a,b}: 0), brute force (A²∘A), t(v) = Σ_{e∋v} support(e) / 2.
  *   orc_cost_eq1         Eq.1 numerator Σ_u |n·d~(u) − m|, exact 128-bit
  *   orc_superiority      S(d) = llround(2^20 (F_m(d) − λ F_c(d))) (Eq.22; Q20)
  *   orc_objective_eq3    Eq.3 Σ_i |Σ_{v∈B_i} S(v)| with λ folded into S
@@ -614,4 +621,23 @@ uint64_t orc_count_forward(uint32_t n, const uint64_t *offs, const uint32_t *col
     }
   }
   return T;
+}
+
+/* ------------------------------------------------------------------------ */
+/* per-edge triangle counts (support)                                        */
+/* ------------------------------------------------------------------------ */
+/* edges: m sorted keys (min << 32) | max; offs/adj: the symmetric CSR of orc_sym_csr
+ * (ascending lists).  out[e] = |N(a) ∩ N(b)| for edge e = {a, b}. */
+void orc_edge_support(const uint64_t *edges, uint64_t m, const uint64_t *offs, const uint32_t *adj,
+                      uint64_t *out) {
+  for (uint64_t e = 0; e < m; ++e) {
+    uint32_t a = (uint32_t)(edges[e] >> 32), b = (uint32_t)(edges[e] & 0xffffffffu);
+    uint64_t i = offs[a], ie = offs[a + 1], j = offs[b], je = offs[b + 1], c = 0;
+    while (i < ie && j < je) {
+      if (adj[i] < adj[j]) ++i;
+      else if (adj[i] > adj[j]) ++j;
+      else { ++c; ++i; ++j; }
+    }
+    out[e] = c;
+  }
 }

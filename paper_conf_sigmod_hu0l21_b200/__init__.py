@@ -78,6 +78,7 @@ def lib():
             "tc_set_schedule": [p, i32],
             "tc_count": [p, p, p],
             "tc_count_range": [p, u32, u32, p, p],
+            "tc_count_edges": [p, p, p],
             "tc_partition": [p, u32, p],
             "tc_nccl_get_unique_id": [p],
             "tc_nccl_comm_init": [p, i32, i32, i32, pp],
@@ -180,6 +181,13 @@ def tc_set_schedule(g, sched):
 def tc_count(g, per_vertex=None):
     T = ctypes.c_uint64()
     _check(lib().tc_count(g, ctypes.byref(T), _ptr(per_vertex)))
+    return T.value
+
+
+def tc_count_edges(g, per_edge):
+    """T and the per-edge triangle counts in canonical edge order (tc_export_graph order)."""
+    T = ctypes.c_uint64()
+    _check(lib().tc_count_edges(g, ctypes.byref(T), _ptr(per_edge)))
     return T.value
 
 
@@ -310,6 +318,13 @@ class Graph:
         t = np.zeros(max(self.n, 1), dtype=np.uint64)
         T = tc_count(self._h, t)
         return T, t[: self.n]
+
+    def count_edges(self):
+        """(T, support[m]): triangles per undirected edge, canonical edge order."""
+        m = int(tc_get_stats(self._h)["m"])
+        te = np.zeros(max(m, 1), dtype=np.uint64)
+        T = tc_count_edges(self._h, te)
+        return T, te[:m]
 
     def count_range(self, u_begin, u_end, per_vertex=False):
         if not per_vertex:

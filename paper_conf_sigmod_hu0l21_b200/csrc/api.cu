@@ -339,6 +339,35 @@ tc_status tc_count(tc_graph *gp, uint64_t *triangles, uint64_t *per_vertex) {
   });
 }
 
+tc_status tc_count_edges(tc_graph *gp, uint64_t *triangles, uint64_t *per_edge) {
+  return guard([&] {
+    Graph &g = checked(gp, G_DIRECTED);
+    TC_REQUIRE(triangles != nullptr, ST_INVALID, "triangles is NULL");
+    TC_REQUIRE(per_edge != nullptr || g.m == 0, ST_INVALID, "per_edge is NULL");
+    StageTimer t(g.stream);
+    ensure_csr(g);
+    cudaStream_t s = g.stream;
+    DevBuf<uint64_t> te, out;
+    te.alloc(g.m ? g.m : 1, s);
+    TC_CUDA(cudaMemsetAsync(te.get(), 0, te.bytes(), s));
+    float kms = 0;
+    uint64_t launches = 0;
+    const uint64_t T = count_graph(g, 0, g.n, te.get(), g_opt_profile ? &kms : nullptr, &launches, 2);
+    if (g.m) {
+      const bool dev = is_device_ptr(per_edge);
+      if (!dev) out.alloc(g.m, s);
+      map_edges_canonical(g, te.get(), dev ? per_edge : out.get());
+      if (!dev) TC_CUDA(cudaMemcpyAsync(per_edge, out.get(), 8ull * g.m, cudaMemcpyDeviceToHost, s));
+    }
+    TC_CUDA(cudaStreamSynchronize(s));
+    g.ms_count = t.stop();
+    g.ms_count_kernel = kms;
+    g.count_launches = launches;
+    g.triangles = T;
+    *triangles = T;
+  });
+}
+
 tc_status tc_count_range(tc_graph *gp, uint32_t u_begin, uint32_t u_end, uint64_t *triangles,
                          uint64_t *per_vertex) {
   return guard([&] {

@@ -80,9 +80,17 @@ __constant__ int g_bracket = 1;  // bracketed binary search on (option "bracket"
 struct GlobalSearch {  // N+(u) in global memory (lists longer than a warp slice)
   const uint32_t *list;
   uint32_t L;
+  uint32_t sbase;  // pos = sbase + index of the last element <= w (per-edge positions)
   __device__ __forceinline__ bool operator()(uint32_t w, uint32_t &pos) const {
-    pos = 0;
-    return bsearch_list(list, L, w);
+    const uint32_t *p = list;
+    uint32_t len = L;
+    while (len > 1) {
+      const uint32_t h = len >> 1;
+      p = (p[h] <= w) ? p + h : p;
+      len -= h;
+    }
+    pos = sbase + (uint32_t)(p - list);
+    return *p == w;
   }
 };
 // Shared-memory loads through 32-bit shared-window byte addresses computed once per
@@ -147,13 +155,20 @@ struct TabSearch {
 // (K entries: start offset, inclusive wedge prefix); each lane walks its owner forward
 // incrementally (its wedge index grows by 32 per step), so locating w's list costs ~1
 // shared load per wedge instead of a 5-step search.
-// Per-vertex mode (PV): matches are first aggregated in shared memory — per owner v in
-// ws.vcnt, per position of w in N+(u) at tc_smem[cbase + pos] — and flushed with one global
-// atomic per distinct vertex per item (hub vertices would otherwise serialise on atomics).
-template <bool PV, class Search>
+// MODE 0: count only.  MODE 1, per-vertex (PV) and MODE 2, per-edge (PE): matches are
+// first aggregated in shared memory — per owner v in ws.vcnt, per position of w in N+(u)
+// at tc_smem[cbase + pos] — and flushed with one global atomic per distinct vertex (PV) or
+// edge (PE) per item (hub vertices would otherwise serialise on atomics).  A triangle
+// u -> v -> w (w in N+(u)) adds one to each of its edges (u,v), (u,w), (v,w) in PE mode:
+// (u,v) through the owner counter, (u,w) through the position counter (or directly at
+// CSR position ebase + index when N+(u) is searched in global memory / a CTA piece), and
+// (v,w) directly at the wedge's own CSR position (unique per wedge).  `tv` is the output:
+// t[n] (PV) or the support of every CSR position (PE).
+template <int MODE, class Search>
 __device__ __forceinline__ uint32_t wedge_loop(const uint32_t *__restrict__ col, const Search &search, uint32_t sbase,
                                                uint32_t cbase, uint32_t lo, uint32_t hi, uint32_t total,
-                                               WarpScratch &ws, unsigned long long *tv) {
+                                               WarpScratch &ws, unsigned long long *tv, uint64_t ebase) {
+  constexpr bool PV = MODE == 1, PE = MODE == 2;
   uint32_t cnt = 0;
   uint32_t o = 0, o_end = ws.pre[0];
   const uint32_t *ob = col + ws.vb[0];  // element j of the current owner list is ob[j]
@@ -166,6 +181,7 @@ __device__ __forceinline__ uint32_t wedge_loop(const uint32_t *__restrict__ col,
   const uint32_t last = total - 1;
   for (uint32_t j0 = lane_id(); j0 < total; j0 += 32 * UNR) {
     uint32_t w[UNR], ow[UNR];
+    uint64_t ep[PE ? UNR : 1];  // PE: CSR position of the wedge's (v, w) edge
 #pragma unroll
     for (int k = 0; k < UNR; ++k) {
       const uint32_t j = min(j0 + 32 * k, last);
@@ -177,16 +193,19 @@ __device__ __forceinline__ uint32_t wedge_loop(const uint32_t *__restrict__ col,
       }
       ow[k] = o;
       w[k] = ldg_u32(ob + j);
+      if (PE) ep[PE ? k : 0] = (uint64_t)(ob - col) + j;
     }
 #pragma unroll
     for (int k = 0; k < UNR; ++k) {
       uint32_t pos;
       const bool hit = search(w[k], pos) && j0 + 32 * k <= last;
       cnt += hit ? 1u : 0u;
-      if (PV && hit) {
+      if ((PV || PE) && hit) {
         atomicAdd(&ws.vcnt[ow[k]], 1u);
         if (cbase != 0xffffffffu) atomicAdd(&tc_smem[cbase + (pos - sbase)], 1u);
-        else atomicAdd(&tv[w[k]], 1ull);
+        else if (PV) atomicAdd(&tv[w[k]], 1ull);
+        else atomicAdd(&tv[ebase + (pos - sbase)], 1ull);
+        if (PE) atomicAdd(&tv[ep[PE ? k : 0]], 1ull);
       }
     }
   }
@@ -220,12 +239,13 @@ __device__ __forceinline__ int build_bracket(uint32_t sbase, uint32_t tbase, uin
 // lies in list[0..L) (w restricted to [lo, hi]).  `padded`: list is the shared-memory copy
 // tc_smem[sbase ..] padded with +inf to 2^ceil(log2 L) (+64) entries; tbase != ~0: room
 // for a bracket table.  Returns this lane's matches.
-template <bool PV>
+template <int MODE>
 __device__ __forceinline__ uint32_t warp_chunk(const uint64_t *__restrict__ offs, const uint32_t *__restrict__ col,
                                                uint32_t v, bool valid, const uint32_t *list, uint32_t sbase,
                                                uint32_t tbase, uint32_t cbase, uint32_t L, bool padded, uint32_t lo,
-                                               uint32_t hi, WarpScratch &ws, unsigned long long *tv, int S2pre = -1,
-                                               uint32_t shpre = 0) {
+                                               uint32_t hi, WarpScratch &ws, unsigned long long *tv, uint32_t vidx,
+                                               uint64_t ua, uint64_t ebase, int S2pre = -1, uint32_t shpre = 0) {
+  constexpr bool PV = MODE == 1, PE = MODE == 2;
   const unsigned lane = lane_id();
   uint64_t vb = 0;
   uint32_t dv = 0;
@@ -241,8 +261,9 @@ __device__ __forceinline__ uint32_t warp_chunk(const uint64_t *__restrict__ offs
     ws.vb[pos] = vb;
     ws.pre[pos] = inc;
     if (PV) ws.v[pos] = v;
+    if (PE) ws.v[pos] = vidx;  // index of v in N+(u): the (u,v) edge is CSR position ua + vidx
   }
-  if (PV) ws.vcnt[lane] = 0;
+  if (PV || PE) ws.vcnt[lane] = 0;
   __syncwarp();
   uint32_t cnt = 0;
   if (total) {
@@ -259,8 +280,8 @@ __device__ __forceinline__ uint32_t warp_chunk(const uint64_t *__restrict__ offs
       switch (S2) {
 #define TC_TAB(k) \
   case k:                                                                                                     \
-    cnt = wedge_loop<PV>(col, TabSearch<k>{smem_addr(sbase), smem_addr(tbase), lo, sh, ((hi - lo) >> sh) + 1, sbase}, \
-                         sbase, cbase, lo, hi, total, ws, tv);                                                \
+    cnt = wedge_loop<MODE>(col, TabSearch<k>{smem_addr(sbase), smem_addr(tbase), lo, sh, ((hi - lo) >> sh) + 1, sbase}, \
+                           sbase, cbase, lo, hi, total, ws, tv, ebase);                                       \
     break;
         TC_TAB(0) TC_TAB(1) TC_TAB(2) TC_TAB(3) TC_TAB(4) TC_TAB(5) TC_TAB(6)
 #undef TC_TAB
@@ -268,17 +289,19 @@ __device__ __forceinline__ uint32_t warp_chunk(const uint64_t *__restrict__ offs
     } else {
       switch (S) {
 #define TC_CASE(k) \
-  case k: cnt = wedge_loop<PV>(col, Pow2Search<k>{smem_addr(sbase), sbase}, sbase, cbase, lo, hi, total, ws, tv); break;
+  case k: cnt = wedge_loop<MODE>(col, Pow2Search<k>{smem_addr(sbase), sbase}, sbase, cbase, lo, hi, total, ws, tv, ebase); break;
         TC_CASE(1) TC_CASE(2) TC_CASE(3) TC_CASE(4) TC_CASE(5) TC_CASE(6) TC_CASE(7)
         TC_CASE(8) TC_CASE(9) TC_CASE(10) TC_CASE(11) TC_CASE(12) TC_CASE(13) TC_CASE(14)
 #undef TC_CASE
         default:
-          cnt = wedge_loop<PV>(col, GlobalSearch{list, L}, sbase, 0xffffffffu, lo, hi, total, ws, tv);
+          cnt = wedge_loop<MODE>(col, GlobalSearch{list, L, sbase}, sbase, 0xffffffffu, lo, hi, total, ws, tv, ebase);
       }
     }
   }
   __syncwarp();
   if (PV && lane < (unsigned)__popc(nz) && ws.vcnt[lane]) atomicAdd(&tv[ws.v[lane]], (unsigned long long)ws.vcnt[lane]);
+  if (PE && lane < (unsigned)__popc(nz) && ws.vcnt[lane])
+    atomicAdd(&tv[ua + ws.v[lane]], (unsigned long long)ws.vcnt[lane]);
   return cnt;
 }
 
@@ -286,23 +309,24 @@ __device__ __forceinline__ uint32_t warp_chunk(const uint64_t *__restrict__ offs
 // warp's shared slice (staged here, padded with +inf to a power of two) when it fits,
 // else in global memory.  Per-warp layout (warp_stride words): slice [cap + 64, +inf
 // padded], bracket table [cap + 64], PV only: match counters [cap].
-template <bool PV>
+template <int MODE>
 __device__ __forceinline__ uint64_t warp_item(const uint64_t *__restrict__ offs, const uint32_t *__restrict__ col,
                                               uint32_t u, uint32_t c0, uint32_t sbase, uint32_t cap,
                                               WarpScratch &ws, unsigned long long *tv) {
+  constexpr bool PV = MODE == 1, PE = MODE == 2;
   const unsigned lane = lane_id();
   const uint64_t a = offs[u];
   const uint32_t L = (uint32_t)(offs[u + 1] - a);
   if (L < 2 || c0 >= L) return 0;
   const uint32_t *list;
   bool padded = false;
-  const uint32_t cbase = (PV && L <= cap) ? sbase + (cap + 64) + (cap + 64) / 2 : 0xffffffffu;
+  const uint32_t cbase = ((PV || PE) && L <= cap) ? sbase + (cap + 64) + (cap + 64) / 2 : 0xffffffffu;
   if (L <= cap) {
     const int SL = ceil_log2(L);
     const uint32_t P = (1u << SL) + (SL >= 6 ? 64u : 0u);  // +64: bracket-search slack
     for (uint32_t j = lane; j < P; j += 32) {
       tc_smem[sbase + j] = j < L ? ldg_u32(col + a + j) : 0xffffffffu;
-      if (PV && j < L) tc_smem[cbase + j] = 0;
+      if ((PV || PE) && j < L) tc_smem[cbase + j] = 0;
     }
     __syncwarp();
     list = tc_smem + sbase;
@@ -313,8 +337,8 @@ __device__ __forceinline__ uint64_t warp_item(const uint64_t *__restrict__ offs,
   const uint32_t lo = list[0], hi = list[L - 1];
   const bool valid = c0 + lane < L;
   const uint32_t v = valid ? list[c0 + lane] : 0u;
-  uint32_t cnt = warp_chunk<PV>(offs, col, v, valid, list, sbase, padded ? sbase + cap + 64 : 0xffffffffu, cbase, L,
-                                padded, lo, hi, ws, tv);
+  uint32_t cnt = warp_chunk<MODE>(offs, col, v, valid, list, sbase, padded ? sbase + cap + 64 : 0xffffffffu, cbase, L,
+                                  padded, lo, hi, ws, tv, c0 + lane, a, a);
   __syncwarp();  // slice reads done before the next item restages it
   if (PV) {
     uint64_t tot = warp_sum((uint64_t)cnt);
@@ -326,6 +350,13 @@ __device__ __forceinline__ uint64_t warp_item(const uint64_t *__restrict__ offs,
       }
       __syncwarp();
     }
+  }
+  if (PE && cbase != 0xffffffffu) {  // (u,w) edges: CSR position a + index of w in N+(u)
+    for (uint32_t j = lane; j < L; j += 32) {
+      const uint32_t c = tc_smem[cbase + j];
+      if (c) atomicAdd(&tv[a + j], (unsigned long long)c);
+    }
+    __syncwarp();
   }
   return cnt;
 }
@@ -417,14 +448,14 @@ __global__ __launch_bounds__(256) void items_scatter_kernel(const uint64_t *__re
 
 // --------------------------------------------------------------- count kernels (a9)
 // Warp items; items [0, nheavy) are fetched one at a time, the rest CHUNK at a time.
-template <bool PV>
+template <int MODE>
 __global__ __launch_bounds__(CT_THREADS, 6) void count_small_kernel(const uint64_t *__restrict__ offs,
                                                                  const uint32_t *__restrict__ col,
                                                                  const uint64_t *__restrict__ items, uint64_t nitems,
                                                                  uint64_t nheavy, unsigned long long *ctr, uint32_t cap,
                                                                  unsigned long long *T, unsigned long long *tv) {
   __shared__ WarpScratch s_ws[CT_WARPS];
-  const uint32_t slice = warp_id() * warp_stride(cap, PV);
+  const uint32_t slice = warp_id() * warp_stride(cap, MODE != 0);
   WarpScratch &ws = s_ws[warp_id()];
   uint64_t acc = 0;
   while (true) {  // heavy items, one per fetch
@@ -433,7 +464,7 @@ __global__ __launch_bounds__(CT_THREADS, 6) void count_small_kernel(const uint64
     i = __shfl_sync(0xffffffffu, i, 0);
     if (i >= nheavy) break;
     uint64_t it = items[i];
-    acc += warp_item<PV>(offs, col, (uint32_t)(it >> 32), (uint32_t)it, slice, cap, ws, tv);
+    acc += warp_item<MODE>(offs, col, (uint32_t)(it >> 32), (uint32_t)it, slice, cap, ws, tv);
   }
   while (true) {  // light items, CHUNK per fetch
     unsigned long long b = 0;
@@ -443,7 +474,7 @@ __global__ __launch_bounds__(CT_THREADS, 6) void count_small_kernel(const uint64
     uint64_t e = min((uint64_t)b + CHUNK, nitems);
     for (uint64_t i = b; i < e; ++i) {
       uint64_t it = items[i];
-      acc += warp_item<PV>(offs, col, (uint32_t)(it >> 32), (uint32_t)it, slice, cap, ws, tv);
+      acc += warp_item<MODE>(offs, col, (uint32_t)(it >> 32), (uint32_t)it, slice, cap, ws, tv);
     }
   }
   block_add_u64(acc, T);
@@ -480,7 +511,7 @@ __device__ __forceinline__ void mbar_wait(uint64_t *bar, unsigned phase) {
 
 // CTA items (u, c0) of heavy sources: v's N+(u)[c0 .. c0+LV) over 16 warps; N+(u) staged
 // piece by piece with a TMA bulk copy (cp.async.bulk + mbarrier complete_tx).
-template <bool PV>
+template <int MODE>
 __global__ __launch_bounds__(LG_THREADS, 5) void count_large_kernel(const uint64_t *__restrict__ offs,
                                                                  const uint32_t *__restrict__ col,
                                                                  const uint64_t *__restrict__ items, uint64_t nitems,
@@ -562,14 +593,14 @@ __global__ __launch_bounds__(LG_THREADS, 5) void count_large_kernel(const uint64
       for (uint32_t c0 = cbeg + warp_id() * 32; c0 < cend; c0 += LG_THREADS) {
         bool valid = c0 + lane_id() < cend;
         uint32_t v = valid ? ldg_u32(col + a + c0 + lane_id()) : 0u;
-        cnt += warp_chunk<PV>(offs, col, v, valid, list, shift, S2 >= 0 ? tbase_lg : 0xffffffffu, 0xffffffffu, plen,
-                              true, lo, hi, ws, tv, S2 >= 0 ? S2 : -2, sh);
+        cnt += warp_chunk<MODE>(offs, col, v, valid, list, shift, S2 >= 0 ? tbase_lg : 0xffffffffu, 0xffffffffu, plen,
+                                true, lo, hi, ws, tv, c0 + lane_id(), a, a + p0, S2 >= 0 ? S2 : -2, sh);
       }
       ucnt += cnt;
       __syncthreads();  // piece fully consumed before the next bulk copy overwrites it
     }
     acc += ucnt;
-    if (PV) {
+    if (MODE == 1) {
       uint64_t tot = warp_sum(ucnt);
       if (lane_id() == 0 && tot) atomicAdd(&tv[u], (unsigned long long)tot);
     }
@@ -578,7 +609,7 @@ __global__ __launch_bounds__(LG_THREADS, 5) void count_large_kernel(const uint64
 }
 
 // RANGE schedule: CTA per bucket of consecutive labels [boff[i], boff[i+1]) ∩ [ub, ue).
-template <bool PV>
+template <int MODE>
 __global__ __launch_bounds__(CT_THREADS) void count_range_kernel(const uint64_t *__restrict__ offs,
                                                                  const uint32_t *__restrict__ col,
                                                                  const uint32_t *__restrict__ boff, uint32_t kfixed,
@@ -587,7 +618,7 @@ __global__ __launch_bounds__(CT_THREADS) void count_range_kernel(const uint64_t 
                                                                  unsigned long long *T, unsigned long long *tv) {
   __shared__ WarpScratch s_ws[CT_WARPS];
   __shared__ uint32_t s_bucket;
-  const uint32_t slice = warp_id() * warp_stride(cap, PV);
+  const uint32_t slice = warp_id() * warp_stride(cap, MODE != 0);
   WarpScratch &ws = s_ws[warp_id()];
   uint64_t acc = 0;
   while (true) {  // buckets fetched dynamically: a CTA takes the next bucket when done
@@ -608,7 +639,7 @@ __global__ __launch_bounds__(CT_THREADS) void count_range_kernel(const uint64_t 
       uint32_t nit = (L + SV - 1) / SV;
       uint32_t first = (warp_id() + CT_WARPS - (t % CT_WARPS)) % CT_WARPS;
       for (uint32_t c = first; c < nit; c += CT_WARPS)
-        acc += warp_item<PV>(offs, col, (uint32_t)u, c * SV, slice, cap, ws, tv);
+        acc += warp_item<MODE>(offs, col, (uint32_t)u, c * SV, slice, cap, ws, tv);
       t += nit;
     }
   }
@@ -619,6 +650,37 @@ __global__ void gather_tv_kernel(const unsigned long long *__restrict__ tnew, co
                                  uint32_t n, uint64_t *__restrict__ out) {
   for (uint64_t v = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (uint64_t)gridDim.x * blockDim.x)
     out[v] = tnew[perm ? perm[v] : v];
+}
+
+// --------------------------------------------------------------- per-edge output order
+__global__ void inverse_perm_kernel(const uint32_t *__restrict__ perm, uint32_t n, uint32_t *__restrict__ iperm) {
+  for (uint64_t v = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (uint64_t)gridDim.x * blockDim.x)
+    iperm[perm[v]] = (uint32_t)v;
+}
+
+// Per-edge support from CSR positions (final labels) to the canonical order of the simple
+// graph's edge list (keys (min << bits) | max over ORIGINAL ids, ascending): one warp per
+// source label, every CSR edge located by a binary search of its canonical key.
+__global__ void edge_map_kernel(const uint64_t *__restrict__ offs, const uint32_t *__restrict__ col, uint32_t n,
+                                const uint32_t *__restrict__ iperm, const uint64_t *__restrict__ edges, uint64_t m,
+                                int bits, const unsigned long long *__restrict__ te, uint64_t *__restrict__ out) {
+  const unsigned warps = gridDim.x * (blockDim.x / 32);
+  for (uint64_t x = (uint64_t)blockIdx.x * (blockDim.x / 32) + warp_id(); x < n; x += warps) {
+    const uint64_t a = offs[x], e = offs[x + 1];
+    const uint32_t ox = iperm ? iperm[x] : (uint32_t)x;
+    for (uint64_t p = a + lane_id(); p < e; p += 32) {
+      const uint32_t y = col[p];
+      const uint32_t oy = iperm ? iperm[y] : y;
+      const uint64_t key = ((uint64_t)min(ox, oy) << bits) | max(ox, oy);
+      uint64_t lo = 0, hi = m;
+      while (lo < hi) {
+        const uint64_t mid = (lo + hi) >> 1;
+        if (edges[mid] < key) lo = mid + 1;
+        else hi = mid;
+      }
+      out[lo] = te[p];
+    }
+  }
 }
 
 // --------------------------------------------------------------- work model / analysis
@@ -671,13 +733,13 @@ static void configure_kernels() {
   static bool done = false;
   if (done) return;
   size_t large_smem = LG_SMEM_WORDS * sizeof(uint32_t);
-  TC_CUDA(cudaFuncSetAttribute(count_large_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)large_smem));
-  TC_CUDA(cudaFuncSetAttribute(count_large_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)large_smem));
+  for (auto fn : {count_large_kernel<0>, count_large_kernel<1>, count_large_kernel<2>})
+    TC_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)large_smem));
   int small_max = 200 * 1024;
-  TC_CUDA(cudaFuncSetAttribute(count_small_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, small_max));
-  TC_CUDA(cudaFuncSetAttribute(count_small_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, small_max));
-  TC_CUDA(cudaFuncSetAttribute(count_range_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, small_max));
-  TC_CUDA(cudaFuncSetAttribute(count_range_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, small_max));
+  for (auto fn : {count_small_kernel<0>, count_small_kernel<1>, count_small_kernel<2>})
+    TC_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, small_max));
+  for (auto fn : {count_range_kernel<0>, count_range_kernel<1>, count_range_kernel<2>})
+    TC_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, small_max));
   done = true;
 }
 
@@ -727,7 +789,9 @@ static int occupancy(const void *fn, int threads, size_t smem) {
   return blocks > 0 ? blocks : 1;
 }
 
-uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *kernel_ms, uint64_t *launches) {
+uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *kernel_ms, uint64_t *launches,
+                     int mode) {
+  if (mode < 0) mode = d_tv ? 1 : 0;  // 0 count, 1 per-vertex (t[n], new labels), 2 per-edge (CSR positions)
   cudaStream_t s = g.stream;
   configure_kernels();
   {
@@ -774,21 +838,17 @@ uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *
         nb = (ue + k - 1) / k - b0;
       }
       if (nb) {
-        size_t smem = (size_t)CT_WARPS * warp_stride(cap, tv != nullptr) * sizeof(uint32_t);
-        int occ = occupancy(tv ? (const void *)count_range_kernel<true> : (const void *)count_range_kernel<false>,
-                            CT_THREADS, smem);
+        size_t smem = (size_t)CT_WARPS * warp_stride(cap, mode != 0) * sizeof(uint32_t);
+        auto range_fn = mode == 2 ? count_range_kernel<2> : mode == 1 ? count_range_kernel<1> : count_range_kernel<0>;
+        int occ = occupancy((const void *)range_fn, CT_THREADS, smem);
         unsigned grid = (unsigned)std::min<uint64_t>(nb, (uint64_t)num_sms() * occ);
         DevBuf<unsigned> bctr;
         bctr.alloc(1, s);
         TC_CUDA(cudaMemsetAsync(bctr.get(), 0, sizeof(unsigned), s));
         if (kernel_ms) TC_CUDA(cudaEventRecord(e0, s));
         ProfScope prof("count_range", s, 0.0);
-        if (tv)
-          count_range_kernel<true><<<grid, CT_THREADS, smem, s>>>(g.offs.get(), g.col.get(), boff, k, b0, nb, ub, ue,
-                                                                   cap, bctr.get(), dT.get(), tv);
-        else
-          count_range_kernel<false><<<grid, CT_THREADS, smem, s>>>(g.offs.get(), g.col.get(), boff, k, b0, nb, ub, ue,
-                                                                    cap, bctr.get(), dT.get(), nullptr);
+        range_fn<<<grid, CT_THREADS, smem, s>>>(g.offs.get(), g.col.get(), boff, k, b0, nb, ub, ue, cap, bctr.get(),
+                                                dT.get(), tv);
         TC_LAUNCH_CHECK();
         if (kernel_ms) TC_CUDA(cudaEventRecord(e1, s));
         ++nlaunch;
@@ -834,35 +894,27 @@ uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *
         if (kernel_ms) TC_CUDA(cudaEventRecord(e0, s));
         if (nlarge) {
           size_t smem = LG_SMEM_WORDS * sizeof(uint32_t);
-          int occ = occupancy(tv ? (const void *)count_large_kernel<true> : (const void *)count_large_kernel<false>,
-                              LG_THREADS, smem);
+          auto large_fn =
+              mode == 2 ? count_large_kernel<2> : mode == 1 ? count_large_kernel<1> : count_large_kernel<0>;
+          int occ = occupancy((const void *)large_fn, LG_THREADS, smem);
           unsigned grid = (unsigned)std::min<uint64_t>(nlarge, (uint64_t)num_sms() * occ);
           ProfScope prof("count_large", s, 0.0);
-          if (tv)
-            count_large_kernel<true><<<grid, LG_THREADS, smem, s>>>(g.offs.get(), g.col.get(), items.get(), nlarge,
-                                                                     hist.get() + 64, dT.get(), tv);
-          else
-            count_large_kernel<false><<<grid, LG_THREADS, smem, s>>>(g.offs.get(), g.col.get(), items.get(), nlarge,
-                                                                      hist.get() + 64, dT.get(), nullptr);
+          large_fn<<<grid, LG_THREADS, smem, s>>>(g.offs.get(), g.col.get(), items.get(), nlarge, hist.get() + 64,
+                                                   dT.get(), tv);
           TC_LAUNCH_CHECK();
           ++nlaunch;
         }
         uint64_t nsmall = nitems - nlarge;
         if (nsmall) {
-          size_t smem = (size_t)CT_WARPS * warp_stride(cap_small, tv != nullptr) * sizeof(uint32_t);
-          int occ = occupancy(tv ? (const void *)count_small_kernel<true> : (const void *)count_small_kernel<false>,
-                              CT_THREADS, smem);
+          size_t smem = (size_t)CT_WARPS * warp_stride(cap_small, mode != 0) * sizeof(uint32_t);
+          auto small_fn =
+              mode == 2 ? count_small_kernel<2> : mode == 1 ? count_small_kernel<1> : count_small_kernel<0>;
+          int occ = occupancy((const void *)small_fn, CT_THREADS, smem);
           uint64_t want = (nsmall + CT_WARPS - 1) / CT_WARPS;
           unsigned grid = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(want, (uint64_t)num_sms() * occ));
           ProfScope prof("count_small", s, 0.0);
-          if (tv)
-            count_small_kernel<true><<<grid, CT_THREADS, smem, s>>>(g.offs.get(), g.col.get(), items.get() + nlarge,
-                                                                     nsmall, nheavy, hist.get() + 65, cap_small,
-                                                                     dT.get(), tv);
-          else
-            count_small_kernel<false><<<grid, CT_THREADS, smem, s>>>(g.offs.get(), g.col.get(), items.get() + nlarge,
-                                                                      nsmall, nheavy, hist.get() + 65, cap_small,
-                                                                      dT.get(), nullptr);
+          small_fn<<<grid, CT_THREADS, smem, s>>>(g.offs.get(), g.col.get(), items.get() + nlarge, nsmall, nheavy,
+                                                   hist.get() + 65, cap_small, dT.get(), tv);
           TC_LAUNCH_CHECK();
           ++nlaunch;
         }
@@ -882,6 +934,21 @@ uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *
   }
   if (launches) *launches = nlaunch;
   return hT;
+}
+
+void map_edges_canonical(Graph &g, const uint64_t *d_te, uint64_t *d_out) {
+  cudaStream_t s = g.stream;
+  if (!g.m) return;
+  DevBuf<uint32_t> iperm;
+  if (!g.identity_perm) {
+    iperm.alloc(g.n, s);
+    inverse_perm_kernel<<<grid_for(g.n, 256), 256, 0, s>>>(g.perm.get(), g.n, iperm.get());
+    TC_LAUNCH_CHECK();
+  }
+  edge_map_kernel<<<grid_for((uint64_t)g.n * 32, 256), 256, 0, s>>>(
+      g.offs.get(), g.col.get(), g.n, g.identity_perm ? nullptr : iperm.get(), g.edges.get(), g.m, g.bits,
+      reinterpret_cast<const unsigned long long *>(d_te), d_out);
+  TC_LAUNCH_CHECK();
 }
 
 void gather_per_vertex(Graph &g, const uint64_t *d_tnew, uint64_t *d_out) {

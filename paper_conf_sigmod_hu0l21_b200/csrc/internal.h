@@ -83,7 +83,9 @@ void aorder_host(const std::vector<uint32_t> &od, const tc_aorder_params &p, std
                  std::vector<uint32_t> &bucket_off, int64_t &eq3);
 // count.cu
 uint64_t count_graph(Graph &g, uint32_t u_begin, uint32_t u_end, uint64_t *d_tv /*new labels or null*/,
-                     float *kernel_ms, uint64_t *launches);
+                     float *kernel_ms, uint64_t *launches, int mode = -1 /*-1: 1 if d_tv else 0; 2 = per-edge*/);
+// per-edge support in CSR positions (final labels) -> canonical order of g.edges (original ids)
+void map_edges_canonical(Graph &g, const uint64_t *d_te, uint64_t *d_out);
 void gather_per_vertex(Graph &g, const uint64_t *d_tnew, uint64_t *d_out);
 void partition_graph(Graph &g, uint32_t world, uint32_t *bounds);
 void analyze_graph(Graph &g);

@@ -153,3 +153,56 @@ def random_graph(rng, n, m_samples, kind="er"):
         src = rng.choice(n, size=m_samples, p=w)
         dst = rng.choice(n, size=m_samples, p=w)
     return src.astype(np.uint32), dst.astype(np.uint32)
+
+
+# Per-edge triangle counts ("support") in closed form, as a function of
+# the builder's own labels (u < v not assumed).
+def _support_wheel(r):
+    if r == 3:
+        return lambda u, v: 2
+    return lambda u, v: 2 if 0 in (u, v) else 1
+
+
+def _support_tripartite(a, b, c):
+    def part(x):
+        return 0 if x < a else (1 if x < a + b else 2)
+    sizes = (a, b, c)
+    return lambda u, v: sizes[3 - part(u) - part(v)]
+
+
+SUPPORT = {
+    "K3": lambda u, v: 1, "K4": lambda u, v: 2, "K7": lambda u, v: 5, "K12": lambda u, v: 10,
+    "K3_4": lambda u, v: 0, "K6_9": lambda u, v: 0,
+    "W3": _support_wheel(3), "W4": _support_wheel(4), "W9": _support_wheel(9),
+    "K2_3_4": _support_tripartite(2, 3, 4), "K5_5_5": _support_tripartite(5, 5, 5),
+    "F1": lambda u, v: 1, "F8": lambda u, v: 1,
+    "B1": lambda u, v: 1, "B10": lambda u, v: 10 if {u, v} == {0, 1} else 1,
+    "C3": lambda u, v: 1, "C4": lambda u, v: 0, "C11": lambda u, v: 0, "star9": lambda u, v: 0,
+    # K_2t minus a perfect matching: common neighbours of u, v = all but u, v and their partners
+    "CP2": lambda u, v: 0, "CP3": lambda u, v: 2, "CP6": lambda u, v: 8,
+    "petersen": lambda u, v: 0,
+}
+
+
+def expected_support(name, edges, n, perm):
+    """Closed-form support in canonical order of the relabelled simple graph (keys
+    (min << 32) | max over perm[]-labels, ascending)."""
+    f = SUPPORT[name]
+    d = {}
+    for u, v in edges:
+        a, b = int(perm[u]), int(perm[v])
+        d[(min(a, b) << 32) | max(a, b)] = f(u, v)
+    keys = sorted(d)
+    return np.array(keys, dtype=np.uint64), np.array([d[k] for k in keys], dtype=np.uint64)
+
+
+def brute_force_support(src, dst, n):
+    """(A @ A) ∘ A on the dense adjacency: common neighbours of every adjacent pair, in
+    canonical (min, max) order."""
+    A = np.zeros((n, n), dtype=np.int64)
+    for u, v in zip(src.tolist(), dst.tolist()):
+        if u != v:
+            A[u, v] = A[v, u] = 1
+    A2 = A @ A
+    iu, iv = np.nonzero(np.triu(A, 1))
+    return ((iu.astype(np.uint64) << np.uint64(32)) | iv.astype(np.uint64)), A2[iu, iv].astype(np.uint64)

@@ -1,10 +1,11 @@
 """Full-size BASELINE.json configs on the GPU, in the launch configuration bench.py times.
 
-* configs[1] (ER, 67M edges): whole oracle vs GPU — oriented CSR bit-exact and T.
+* configs[1] (ER, 67M edges): whole oracle vs GPU — oriented CSR bit-exact, T, per-edge support.
 * configs[2] (R-MAT s22): A-direction orientation bit-exact vs the sequential oracle
   (sub, dsnap, CSR); T equal over ID/degree/A-direction; oracle counts on sampled vertex
   ranges; per-vertex t(v) on sampled vertices vs the oracle's definition straight from
-  the raw samples; Σt = 3T; GPU partition bounds vs the restated work rule.
+  the raw samples; Σt = 3T; GPU partition bounds vs the restated work rule; per-edge
+  support on sampled edges, Σ = 3T.
 * configs[3] (R-MAT s24 ef32): T equal over none/D-order/A-order; sampled t(v); Σt = 3T.
 * configs[4] (Kronecker s27, 2^31 samples): marked slow; same properties.
 """
@@ -46,6 +47,11 @@ def test_config2_er_full_oracle():
     offs, col, perm = g.export()
     assert np.array_equal(offs, ref["offs"]) and np.array_equal(col, ref["col"])
     assert g.count() == ref["T"]
+    # per-edge support (f1), every edge: the oracle's common-neighbour merge on the
+    # symmetric lists vs the GPU's three aggregated increments per triangle
+    T, te = g.count_edges()
+    assert T == ref["T"]
+    assert np.array_equal(te, oracle.edge_support(ref["edges"], spec.n))
     g.free()
 
 
@@ -77,6 +83,12 @@ def test_config3_rmat_s22():
     # work-balanced partition = the restated rule (tests/test_dist_gloo.py)
     for world in (2, 4, 8):
         assert g.partition(world).tolist() == work_bounds_fast(offs, col, world)
+    # per-edge support (f1): Σ = 3T, and uniformly sampled edges (chosen without looking at
+    # the GPU output) against the oracle's common-neighbour merge
+    Te, te = g.count_edges()
+    assert Te == T and int(te.sum()) == 3 * T
+    idx = np.sort(rng.choice(len(edges), size=3000, replace=False))
+    assert np.array_equal(te[idx], oracle.edge_support(edges, n, subset=edges[idx]))
     g.free()
     # T does not depend on the directing rule
     for d in ("id", "degree"):

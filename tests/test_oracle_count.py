@@ -103,3 +103,46 @@ def test_local_triangles_matches_per_vertex():
     s2, d2 = graphs.random_graph(rng, n, 300, "skew")
     _, tv = graphs.brute_force(s2, d2, n)
     assert np.array_equal(oracle.local_triangles(s2, d2, np.arange(n)).astype(np.int64), tv)
+
+
+# ---------------------------------------------------------------- per-edge support (f1)
+@pytest.mark.parametrize("name", sorted(graphs.CLOSED_FORMS))
+def test_edge_support_closed_forms(name):
+    """support(e) = #triangles containing e, against the closed form of every family."""
+    edges, n, T, t = graphs.CLOSED_FORMS[name]
+    rng = np.random.default_rng(zlib.crc32(name.encode()) + 1)
+    src, dst, N, perm = graphs.noisy_samples(edges, n, rng, pad=2)
+    keys, expect = graphs.expected_support(name, edges, n, perm)
+    res = oracle.run(src, dst, N, "degree", "none", per_edge=True)
+    assert np.array_equal(res["edges"], keys)
+    assert np.array_equal(res["te"], expect), name
+    assert int(res["te"].sum()) == 3 * T
+
+
+@pytest.mark.parametrize("seed", range(10))
+def test_edge_support_brute_force(seed):
+    """(A @ A) ∘ A on tiny random graphs (a dropped or double-counted triangle edge fails)."""
+    rng = np.random.default_rng(100 + seed)
+    n = int(rng.integers(2, 60))
+    src, dst = graphs.random_graph(rng, n, int(rng.integers(0, 5 * n)), "er" if seed % 2 else "skew")
+    keys, sup = graphs.brute_force_support(src, dst, n)
+    res = oracle.run(src, dst, n, "id", "none", per_edge=True)
+    assert np.array_equal(res["edges"], keys)
+    assert np.array_equal(res["te"], sup)
+
+
+def test_edge_support_vertex_identity():
+    """Each triangle at v contains exactly two edges at v: t(v) = Σ_{e ∋ v} support(e) / 2,
+    and Σ_e support(e) = 3T (R-MAT scale 10, skewed)."""
+    import graphgen
+    spec = graphgen.rmat_spec(10, 16, 7)
+    src, dst = graphgen.generate_cpu(spec)
+    res = oracle.run(src, dst, spec.n, "degree", "none", per_vertex=True, per_edge=True)
+    te = res["te"].astype(np.int64)
+    assert int(te.sum()) == 3 * res["T"]
+    a = (res["edges"] >> np.uint64(32)).astype(np.int64)
+    b = (res["edges"] & np.uint64(0xffffffff)).astype(np.int64)
+    acc = np.zeros(spec.n, dtype=np.int64)
+    np.add.at(acc, a, te)
+    np.add.at(acc, b, te)
+    assert np.array_equal(acc // 2, res["t"].astype(np.int64)) and not (acc % 2).any()
