@@ -183,6 +183,10 @@ tc_status tc_set_option(const char *key, int64_t value) {
     else if (k == "l2_persist") g_opt_l2_persist = value ? 1 : 0;
     else if (k == "trim_memory") dev_trim();
     else if (k == "bracket") g_opt_bracket = value ? 1 : 0;
+    else if (k == "intersect") {
+      TC_REQUIRE(value == 0 || value == 1, ST_INVALID, "intersect: 0 = binary search, 1 = sort-merge");
+      g_opt_intersect = (int)value;
+    }
     else if (k == "peel_coop") g_opt_peel_coop = value ? 1 : 0;
     else if (k == "split") g_opt_split = value ? 1 : 0;
     else if (k == "small_cap") {

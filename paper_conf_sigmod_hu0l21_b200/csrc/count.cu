@@ -29,6 +29,7 @@ namespace tc {
 
 int g_opt_small_cap = 256;   // power of two: d~ below it -> warp items, else CTA items
 int g_opt_bracket = 1;       // bracketed binary search for long staged lists
+int g_opt_intersect = 0;     // 0 = binary search (the paper's kernel), 1 = sort-merge (P:548-550 comparison)
 int g_opt_l2_persist = 0;    // L2 access-policy window over [offs | col] during counts (off: measured slower overall)
 
 namespace {
@@ -75,6 +76,34 @@ __host__ __device__ constexpr uint32_t warp_stride(uint32_t cap, bool pv) {
 }
 
 __constant__ int g_bracket = 1;  // bracketed binary search on (option "bracket")
+__constant__ int g_merge = 0;    // sort-merge intersection instead of binary search (option "intersect")
+
+// Sort-merge intersection (the strategy the paper compares binary search against, §6.2,
+// P:548-550, Fig.10): lane l intersects N+(u) (`list`, ascending, shared or global) with
+// its own N+(v) (col[vb .. vb+dv), ascending) by a two-pointer merge.  Every lane walks
+// its own pair of lists, so a warp runs as long as its longest merge (the divergence the
+// paper's argument for binary search rests on).  Count only.
+__device__ __forceinline__ uint32_t merge_lane(const uint32_t *list, uint32_t L, const uint32_t *__restrict__ B,
+                                               uint32_t dv) {
+  uint32_t cnt = 0;
+  if (dv == 0 || L == 0) return 0;
+  uint32_t i = 0, j = 0, a = list[0], b = __ldg(B);
+  while (true) {
+    if (a < b) {
+      if (++i == L) break;
+      a = list[i];
+    } else if (a > b) {
+      if (++j == dv) break;
+      b = __ldg(B + j);
+    } else {
+      ++cnt;
+      if (++i == L || ++j == dv) break;
+      a = list[i];
+      b = __ldg(B + j);
+    }
+  }
+  return cnt;
+}
 
 // Searchers: does w occur in N+(u)?  `pos` = its shared-memory index (PV counters).
 struct GlobalSearch {  // N+(u) in global memory (lists longer than a warp slice)
@@ -266,6 +295,7 @@ __device__ __forceinline__ uint32_t warp_chunk(const uint64_t *__restrict__ offs
   if (PV || PE) ws.vcnt[lane] = 0;
   __syncwarp();
   uint32_t cnt = 0;
+  if (MODE == 0 && g_merge) return merge_lane(list, L, col + vb, dv);
   if (total) {
     const int S = padded ? ceil_log2(L) : 0;
     int S2 = S2pre >= 0 ? S2pre : 99;  // S2pre: table prebuilt by the CTA (large kernel)
@@ -795,10 +825,14 @@ uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *
   cudaStream_t s = g.stream;
   configure_kernels();
   {
-    static int last_bracket = 1;
+    static int last_bracket = 1, last_intersect = 0;
     if (g_opt_bracket != last_bracket) {
       TC_CUDA(cudaMemcpyToSymbol(g_bracket, &g_opt_bracket, sizeof(int)));
       last_bracket = g_opt_bracket;
+    }
+    if (g_opt_intersect != last_intersect) {
+      TC_CUDA(cudaMemcpyToSymbol(g_merge, &g_opt_intersect, sizeof(int)));
+      last_intersect = g_opt_intersect;
     }
   }
   if (ue > g.n) ue = g.n;

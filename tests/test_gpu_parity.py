@@ -362,3 +362,33 @@ def test_count_edges_config1_and_device_output():
         assert np.array_equal(out.cpu().numpy().astype(np.uint64), ref["te"])
     finally:
         g.free()
+
+
+# ---------------------------------------------------------------- sort-merge intersection (§6.2)
+@pytest.mark.parametrize("sched", ["bucketed", "range"])
+@pytest.mark.parametrize("cap", [32, 256, 2048])
+def test_sort_merge_intersection(sched, cap):
+    """The sort-merge variant of the paper's §6.2 comparison (option "intersect"=1) counts
+    the same T on every kernel path (warp slices, global lists, CTA pieces)."""
+    tc.tc_set_option("small_cap", cap)
+    tc.tc_set_option("intersect", 1)
+    try:
+        for seed, (sc, ef) in enumerate(((12, 16), (13, 8))):
+            spec = graphgen.rmat_spec(sc, ef, 90 + seed)
+            src, dst = graphgen.generate_cpu(spec)
+            ref = oracle.run(src, dst, spec.n, "id", "none")
+            for d, r in (("id", "none"), ("degree", "degree"), ("paper", "paper")):
+                g = tc.Graph(src, dst, spec.n).direct(d).reorder(r).set_schedule(sched)
+                assert g.count() == ref["T"], (d, r)
+                T, t = g.count(per_vertex=True)  # per-vertex stays on binary search
+                assert T == ref["T"]
+                g.free()
+        for name in ("K12", "W9", "B10", "CP6", "petersen"):
+            edges, n, T, t = graphs.CLOSED_FORMS[name]
+            src, dst, N, perm = graphs.noisy_samples(edges, n, np.random.default_rng(3), pad=2)
+            g = tc.Graph(src, dst, N).direct("degree").set_schedule(sched)
+            assert g.count() == T, name
+            g.free()
+    finally:
+        tc.tc_set_option("intersect", 0)
+        tc.tc_set_option("small_cap", 256)

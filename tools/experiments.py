@@ -22,6 +22,7 @@ def main():
     ap.add_argument("--rules", default="id:none,degree:none,paper:none,degree:degree,degree:paper,paper:paper")
     ap.add_argument("--schedules", default="bucketed,range")
     ap.add_argument("--reps", type=int, default=3)
+    ap.add_argument("--intersect", default="0", help="comma list: 0 binary search, 1 sort-merge (§6.2)")
     a = ap.parse_args()
     spec = graphgen.CONFIGS[a.config]
     src = torch.empty(spec.samples, dtype=torch.int32, device="cuda")
@@ -29,13 +30,14 @@ def main():
     graphgen.generate_cuda(spec, src.data_ptr(), dst.data_ptr(), torch.cuda.current_stream().cuda_stream)
     torch.cuda.synchronize()
     print(f"### {spec.name} (BASELINE configs[{a.config - 1}]), device ms (median of {a.reps})\n")
-    print("| directing | ordering | schedule | build | direct | reorder | count | total | count GTEPS | total GTEPS "
-          "| max d~ | Eq.1 n*C | Eq.3 | T |")
-    print("|---|---|---|---|---|---|---|---|---|---|---|---|---|---|")
+    print("| directing | ordering | schedule | intersect | build | direct | reorder | count | total | count GTEPS "
+          "| total GTEPS | max d~ | Eq.1 n*C | Eq.3 | T |")
+    print("|---|---|---|---|---|---|---|---|---|---|---|---|---|---|---|")
     prm, keep = tc.make_aorder_params()
     for rule in a.rules.split(","):
         d, r = rule.split(":")
-        for sched in a.schedules.split(","):
+        for sched, isect in [(x, y) for x in a.schedules.split(",") for y in a.intersect.split(",")]:
+            tc.tc_set_option("intersect", int(isect))
             rows = []
             for rep in range(a.reps + 1):
                 g = tc.Graph(src, dst, spec.n)
@@ -50,7 +52,7 @@ def main():
             med = {k: statistics.median(x[k] for x in rows) for k in ("ms_build", "ms_direct", "ms_reorder", "ms_count")}
             tot = sum(med.values())
             m = st["m"]
-            print(f"| {d} | {r} | {sched} | {med['ms_build']:.2f} | {med['ms_direct']:.2f} | {med['ms_reorder']:.2f} | "
+            print(f"| {d} | {r} | {sched} | {'sort-merge' if isect == '1' else 'binary search'} | {med['ms_build']:.2f} | {med['ms_direct']:.2f} | {med['ms_reorder']:.2f} | "
                   f"{med['ms_count']:.2f} | {tot:.2f} | {m / med['ms_count'] / 1e6:.2f} | {m / tot / 1e6:.2f} | "
                   f"{st['max_outdeg']} | {st['eq1']} | {st['eq3']} | {T} |", flush=True)
 
