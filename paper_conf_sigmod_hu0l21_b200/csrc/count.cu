@@ -193,51 +193,65 @@ struct TabSearch {
 // CSR position ebase + index when N+(u) is searched in global memory / a CTA piece), and
 // (v,w) directly at the wedge's own CSR position (unique per wedge).  `tv` is the output:
 // t[n] (PV) or the support of every CSR position (PE).
+// N consecutive 32-wedge steps of one lane (j0, j0 + 32, ...): the N loads are issued back
+// to back before any search (memory-level parallelism for the gather; the owner walk stays
+// incremental).  The tail is branch-free: indices past `last` are clamped to the last wedge
+// (a valid address) and their hits masked (a clamped w must not count twice; +inf would
+// match the padding).
+template <int N, int MODE, class Search>
+__device__ __forceinline__ void wedge_block(uint32_t j0, uint32_t last, const uint32_t *__restrict__ col,
+                                            const Search &search, WarpScratch &ws, uint32_t &o, uint32_t &o_end,
+                                            const uint32_t *&ob, uint32_t &cnt, uint32_t sbase, uint32_t cbase,
+                                            unsigned long long *tv, uint64_t ebase) {
+  constexpr bool PV = MODE == 1, PE = MODE == 2;
+  uint32_t w[N], ow[N];
+  uint64_t ep[PE ? N : 1];  // PE: CSR position of the wedge's (v, w) edge
+#pragma unroll
+  for (int k = 0; k < N; ++k) {
+    const uint32_t j = min(j0 + 32 * k, last);
+    while (o_end <= j) {
+      const uint32_t o_beg = o_end;
+      ++o;
+      o_end = ws.pre[o];
+      ob = col + ws.vb[o] - o_beg;
+    }
+    ow[k] = o;
+    w[k] = ldg_u32(ob + j);
+    if (PE) ep[PE ? k : 0] = (uint64_t)(ob - col) + j;
+  }
+#pragma unroll
+  for (int k = 0; k < N; ++k) {
+    uint32_t pos;
+    const bool hit = search(w[k], pos) && j0 + 32 * k <= last;
+    cnt += hit ? 1u : 0u;
+    if ((PV || PE) && hit) {
+      atomicAdd(&ws.vcnt[ow[k]], 1u);
+      if (cbase != 0xffffffffu) atomicAdd(&tc_smem[cbase + (pos - sbase)], 1u);
+      else if (PV) atomicAdd(&tv[w[k]], 1ull);
+      else atomicAdd(&tv[ebase + (pos - sbase)], 1ull);
+      if (PE) atomicAdd(&tv[ep[PE ? k : 0]], 1ull);
+    }
+  }
+}
+
+// All wedges of one chunk: blocks of 4 steps, then a 2- and a 1-step block for the rest
+// (an ER item has ~5 steps: 4 + 1 slots instead of 8).
 template <int MODE, class Search>
 __device__ __forceinline__ uint32_t wedge_loop(const uint32_t *__restrict__ col, const Search &search, uint32_t sbase,
                                                uint32_t cbase, uint32_t lo, uint32_t hi, uint32_t total,
                                                WarpScratch &ws, unsigned long long *tv, uint64_t ebase) {
-  constexpr bool PV = MODE == 1, PE = MODE == 2;
   uint32_t cnt = 0;
   uint32_t o = 0, o_end = ws.pre[0];
   const uint32_t *ob = col + ws.vb[0];  // element j of the current owner list is ob[j]
-  // UNR wedges per lane in flight: their loads are issued back to back before any search
-  // (memory-level parallelism for the gather; the owner walk stays incremental).  The
-  // tail is branch-free: indices past `total` are clamped to the last wedge (a valid
-  // address) and their hits masked (a clamped w must not count twice; +inf would match
-  // the padding).
-  constexpr int UNR = 4;
-  const uint32_t last = total - 1;
-  for (uint32_t j0 = lane_id(); j0 < total; j0 += 32 * UNR) {
-    uint32_t w[UNR], ow[UNR];
-    uint64_t ep[PE ? UNR : 1];  // PE: CSR position of the wedge's (v, w) edge
-#pragma unroll
-    for (int k = 0; k < UNR; ++k) {
-      const uint32_t j = min(j0 + 32 * k, last);
-      while (o_end <= j) {
-        const uint32_t o_beg = o_end;
-        ++o;
-        o_end = ws.pre[o];
-        ob = col + ws.vb[o] - o_beg;
-      }
-      ow[k] = o;
-      w[k] = ldg_u32(ob + j);
-      if (PE) ep[PE ? k : 0] = (uint64_t)(ob - col) + j;
-    }
-#pragma unroll
-    for (int k = 0; k < UNR; ++k) {
-      uint32_t pos;
-      const bool hit = search(w[k], pos) && j0 + 32 * k <= last;
-      cnt += hit ? 1u : 0u;
-      if ((PV || PE) && hit) {
-        atomicAdd(&ws.vcnt[ow[k]], 1u);
-        if (cbase != 0xffffffffu) atomicAdd(&tc_smem[cbase + (pos - sbase)], 1u);
-        else if (PV) atomicAdd(&tv[w[k]], 1ull);
-        else atomicAdd(&tv[ebase + (pos - sbase)], 1ull);
-        if (PE) atomicAdd(&tv[ep[PE ? k : 0]], 1ull);
-      }
-    }
+  const uint32_t last = total - 1, steps = (total + 31) >> 5, lane = lane_id();
+  uint32_t st = 0;
+  for (; st + 4 <= steps; st += 4)
+    wedge_block<4, MODE>(lane + 32 * st, last, col, search, ws, o, o_end, ob, cnt, sbase, cbase, tv, ebase);
+  if (st + 2 <= steps) {
+    wedge_block<2, MODE>(lane + 32 * st, last, col, search, ws, o, o_end, ob, cnt, sbase, cbase, tv, ebase);
+    st += 2;
   }
+  if (st < steps) wedge_block<1, MODE>(lane + 32 * st, last, col, search, ws, o, o_end, ob, cnt, sbase, cbase, tv, ebase);
   (void)lo;
   (void)hi;
   return cnt;
@@ -479,7 +493,7 @@ __global__ __launch_bounds__(256) void items_scatter_kernel(const uint64_t *__re
 // --------------------------------------------------------------- count kernels (a9)
 // Warp items; items [0, nheavy) are fetched one at a time, the rest CHUNK at a time.
 template <int MODE>
-__global__ __launch_bounds__(CT_THREADS, 6) void count_small_kernel(const uint64_t *__restrict__ offs,
+__global__ __launch_bounds__(CT_THREADS, MODE == 0 ? 6 : 4) void count_small_kernel(const uint64_t *__restrict__ offs,
                                                                  const uint32_t *__restrict__ col,
                                                                  const uint64_t *__restrict__ items, uint64_t nitems,
                                                                  uint64_t nheavy, unsigned long long *ctr, uint32_t cap,
