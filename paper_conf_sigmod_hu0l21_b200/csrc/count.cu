@@ -39,7 +39,10 @@ constexpr int CT_WARPS = CT_THREADS / 32;
 constexpr int LG_THREADS = 256;       // large kernel: 8 warps
 constexpr int LG_WARPS = LG_THREADS / 32;
 constexpr uint32_t PIECE = 4096;      // large kernel: N+(u) piece in shared memory (16 KB)
-constexpr uint32_t LG_SMEM_WORDS = (PIECE + 72) + (PIECE + 64) / 2;  // piece (+pad) + u16 bracket table
+// bracket tables get 2^TS_* buckets per list element (finer buckets: fewer search steps)
+constexpr int TS_W = 2;               // warp items
+constexpr int TS_L = 1;               // CTA items (pieces)
+constexpr uint32_t LG_SMEM_WORDS = (PIECE + 72) + ((PIECE << TS_L) + 64) / 2;  // piece (+pad) + u16 table
 constexpr uint32_t CHUNK = 8;         // worklist entries per atomic fetch
 
 struct WarpScratch {  // per-warp owner-search tables for one 32-v chunk
@@ -71,8 +74,9 @@ __device__ __forceinline__ int ceil_log2(uint32_t L) { return L <= 1 ? 0 : 32 - 
 
 // words of dynamic shared memory per warp in the warp-item kernels
 // (slice cap+64 words, u16 bracket table cap+64 entries, PV counters cap words)
+__host__ __device__ constexpr uint32_t tab_words(uint32_t cap) { return ((cap << TS_W) + 64) / 2; }
 __host__ __device__ constexpr uint32_t warp_stride(uint32_t cap, bool pv) {
-  return (cap + 64) + (cap + 64) / 2 + (pv ? cap : 0);
+  return (cap + 64) + tab_words(cap) + (pv ? cap : 0);
 }
 
 __constant__ int g_bracket = 1;  // bracketed binary search on (option "bracket")
@@ -316,7 +320,7 @@ __device__ __forceinline__ uint32_t warp_chunk(const uint64_t *__restrict__ offs
     uint32_t sh = shpre;
     if (S2pre < 0 && S >= 6 && tbase != 0xffffffffu && g_bracket && total >= 2 * L) {
       const int span_bits = 32 - __clz(hi - lo);  // bits of (hi - lo)
-      sh = span_bits > S ? (uint32_t)(span_bits - S) : 0u;
+      sh = span_bits > S + TS_W ? (uint32_t)(span_bits - S - TS_W) : 0u;
       S2 = build_bracket(sbase, tbase, L, lo, hi, sh);
       __syncwarp();
     }
@@ -364,7 +368,7 @@ __device__ __forceinline__ uint64_t warp_item(const uint64_t *__restrict__ offs,
   if (L < 2 || c0 >= L) return 0;
   const uint32_t *list;
   bool padded = false;
-  const uint32_t cbase = ((PV || PE) && L <= cap) ? sbase + (cap + 64) + (cap + 64) / 2 : 0xffffffffu;
+  const uint32_t cbase = ((PV || PE) && L <= cap) ? sbase + (cap + 64) + tab_words(cap) : 0xffffffffu;
   if (L <= cap) {
     const int SL = ceil_log2(L);
     const uint32_t P = (1u << SL) + (SL >= 6 ? 64u : 0u);  // +64: bracket-search slack
@@ -612,7 +616,7 @@ __global__ __launch_bounds__(LG_THREADS, 5) void count_large_kernel(const uint64
       const int S = ceil_log2(plen);
       if (g_bracket && S >= 6) {
         const int span_bits = 32 - __clz(hi - lo);
-        sh = span_bits > S ? (uint32_t)(span_bits - S) : 0u;
+        sh = span_bits > S + TS_L ? (uint32_t)(span_bits - S - TS_L) : 0u;
         const uint32_t B = ((hi - lo) >> sh) + 1;
         uint16_t *tab = reinterpret_cast<uint16_t *>(tc_smem + tbase_lg);
         for (uint32_t j = threadIdx.x; j < plen; j += LG_THREADS) {
