@@ -180,7 +180,9 @@ tc_status tc_export_buckets(tc_graph *g, uint32_t *bucket_off);
  * oriented CSR by splitting the sorted edge list into forward and reversed runs and sorting
  * only the reversed run, default 1; 0 = sort every oriented key), "intersect" (0 = binary
  * search, the paper's kernel, default; 1 = sort-merge: each lane two-pointer-merges N+(u)
- * with its N+(v), the strategy of the paper's §6.2 comparison; applies to
+ * with its N+(v), the strategy of the paper's §6.2 comparison; 2 = bitmap:
+ * Bisson's block-per-vertex pattern, N+(u) marked in a |V|-bit bitmap, one thread per v
+ * per barrier-closed superstep, the kernel of Fig.13; 1 and 2 apply to
  * tc_count / tc_count_range / tc_count_dist without per-vertex output), "peel_coop" (0/1:
  * run the whole A-direction peel as one cooperative launch with grid-wide barriers instead
  * of 5 launches and a host round trip per subround, default 1), "trim_memory" (any

@@ -184,7 +184,7 @@ tc_status tc_set_option(const char *key, int64_t value) {
     else if (k == "trim_memory") dev_trim();
     else if (k == "bracket") g_opt_bracket = value ? 1 : 0;
     else if (k == "intersect") {
-      TC_REQUIRE(value == 0 || value == 1, ST_INVALID, "intersect: 0 = binary search, 1 = sort-merge");
+      TC_REQUIRE(value >= 0 && value <= 2, ST_INVALID, "intersect: 0 = binary search, 1 = sort-merge, 2 = bitmap");
       g_opt_intersect = (int)value;
     }
     else if (k == "peel_coop") g_opt_peel_coop = value ? 1 : 0;

@@ -694,6 +694,67 @@ __global__ __launch_bounds__(CT_THREADS) void count_range_kernel(const uint64_t 
   block_add_u64(acc, T);
 }
 
+// Bitmap intersection (option "intersect" = 2): Bisson's block-per-vertex pattern as the
+// paper describes it (Fig.1) and evaluates A-direction on (Fig.13):
+// the CTA marks N+(u) in a bitmap of |V| bits, synchronises, then in supersteps of
+// BM_THREADS neighbours each thread takes one v in N+(u) and tests every w in N+(v)
+// against the bitmap; a barrier closes every superstep, so a superstep lasts as long as
+// its longest N+(v) — the intra-block BSP imbalance Eq.1 models.  The bits of
+// N+(u) are cleared again before the next u.  Bitmap in shared memory when |V| <= 2^20
+// (128 KB), else one |V|-bit slice of global memory per CTA (L2-resident for |V| = 2^22).
+constexpr int BM_THREADS = 256;
+constexpr uint32_t BM_CHUNK = 16;  // sources per counter fetch
+constexpr uint32_t BM_SMEM_MAX_N = 1u << 20;
+template <bool SMEM>
+__global__ __launch_bounds__(BM_THREADS) void count_bitmap_kernel(const uint64_t *__restrict__ offs,
+                                                                  const uint32_t *__restrict__ col, uint32_t ub,
+                                                                  uint32_t ue, uint32_t *gbits, uint32_t words,
+                                                                  unsigned *ctr, unsigned long long *T) {
+  uint32_t *bits = SMEM ? tc_smem : gbits + (uint64_t)blockIdx.x * words;
+  __shared__ uint32_t s_c;
+  if (SMEM)
+    for (uint32_t i = threadIdx.x; i < words; i += BM_THREADS) bits[i] = 0u;
+  uint64_t acc = 0;
+  const uint32_t nu = ue - ub;
+  while (true) {
+    __syncthreads();
+    if (threadIdx.x == 0) s_c = atomicAdd(ctr, BM_CHUNK);
+    __syncthreads();
+    const uint32_t c0 = s_c;
+    if (c0 >= nu) break;
+    const uint32_t c1 = min(nu, c0 + BM_CHUNK);
+    for (uint32_t c = c0; c < c1; ++c) {
+      const uint32_t u = ub + c;
+      const uint64_t a = offs[u];
+      const uint32_t L = (uint32_t)(offs[u + 1] - a);
+      if (L < 2) continue;  // block-uniform
+      for (uint32_t i = threadIdx.x; i < L; i += BM_THREADS) {
+        const uint32_t w = __ldg(col + a + i);
+        atomicOr(&bits[w >> 5], 1u << (w & 31));
+      }
+      __syncthreads();
+      uint32_t cnt = 0;
+      for (uint32_t g0 = 0; g0 < L; g0 += BM_THREADS) {  // one superstep per group of neighbours
+        const uint32_t i = g0 + threadIdx.x;
+        if (i < L) {
+          const uint32_t v = __ldg(col + a + i);
+          const uint64_t vb = offs[v];
+          const uint32_t dv = (uint32_t)(offs[v + 1] - vb);
+          for (uint32_t j = 0; j < dv; ++j) {
+            const uint32_t w = __ldg(col + vb + j);
+            cnt += (bits[w >> 5] >> (w & 31)) & 1u;
+          }
+        }
+        __syncthreads();
+      }
+      acc += cnt;
+      for (uint32_t i = threadIdx.x; i < L; i += BM_THREADS) bits[__ldg(col + a + i) >> 5] = 0u;
+      __syncthreads();
+    }
+  }
+  block_add_u64(acc, T);
+}
+
 __global__ void gather_tv_kernel(const unsigned long long *__restrict__ tnew, const uint32_t *__restrict__ perm,
                                  uint32_t n, uint64_t *__restrict__ out) {
   for (uint64_t v = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (uint64_t)gridDim.x * blockDim.x)
@@ -788,6 +849,8 @@ static void configure_kernels() {
     TC_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, small_max));
   for (auto fn : {count_range_kernel<0>, count_range_kernel<1>, count_range_kernel<2>})
     TC_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, small_max));
+  TC_CUDA(cudaFuncSetAttribute(count_bitmap_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                               (int)(BM_SMEM_MAX_N / 8)));
   done = true;
 }
 
@@ -831,6 +894,14 @@ struct L2Window {
   }
 };
 
+// Largest warp-slice capacity <= cap whose per-CTA shared memory (slices, bracket tables,
+// per-vertex/per-edge counters) fits the 200 KB the warp kernels are configured for; lists
+// longer than the slice are searched in global memory (the kernels' L > cap path).
+static uint32_t fit_cap(uint32_t cap, bool pv) {
+  while (cap > 32 && (size_t)CT_WARPS * warp_stride(cap, pv) * sizeof(uint32_t) > 200u * 1024u) cap >>= 1;
+  return cap;
+}
+
 static int occupancy(const void *fn, int threads, size_t smem) {
   int blocks = 0;
   TC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&blocks, fn, threads, smem));
@@ -871,7 +942,32 @@ uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *
     TC_CUDA(cudaEventCreate(&e1));
   }
   L2Window l2win(s, g.csr_mem.get(), g.csr_mem.bytes());
-  if (ub < ue && g.m) {
+  if (ub < ue && g.m && mode == 0 && g_opt_intersect == 2) {
+    // bitmap intersection (Bisson's block-per-vertex pattern): its own schedule
+    const bool in_smem = g.n <= BM_SMEM_MAX_N;
+    const uint32_t words = (g.n + 31) / 32;
+    const size_t smem = in_smem ? (size_t)words * sizeof(uint32_t) : 0;
+    auto fn = in_smem ? count_bitmap_kernel<true> : count_bitmap_kernel<false>;
+    int occ = occupancy((const void *)fn, BM_THREADS, smem);
+    uint64_t want = ((uint64_t)(ue - ub) + BM_CHUNK - 1) / BM_CHUNK;
+    uint64_t grid = std::max<uint64_t>(1, std::min<uint64_t>(want, (uint64_t)num_sms() * occ));
+    DevBuf<uint32_t> gbits;
+    if (!in_smem) {  // one zeroed |V|-bit slice per CTA, at most 1 GiB in total
+      grid = std::max<uint64_t>(1, std::min<uint64_t>(grid, (1ull << 28) / words));
+      gbits.alloc(grid * words, s);
+      TC_CUDA(cudaMemsetAsync(gbits.get(), 0, gbits.bytes(), s));
+    }
+    DevBuf<unsigned> ctr;
+    ctr.alloc(1, s);
+    TC_CUDA(cudaMemsetAsync(ctr.get(), 0, sizeof(unsigned), s));
+    if (kernel_ms) TC_CUDA(cudaEventRecord(e0, s));
+    ProfScope prof("count_bitmap", s, 0.0);
+    fn<<<(unsigned)grid, BM_THREADS, smem, s>>>(g.offs.get(), g.col.get(), ub, ue, gbits.get(), words, ctr.get(),
+                                                 dT.get());
+    TC_LAUNCH_CHECK();
+    if (kernel_ms) TC_CUDA(cudaEventRecord(e1, s));
+    ++nlaunch;
+  } else if (ub < ue && g.m) {
     if (sched == TC_SCHED_RANGE) {
       const uint32_t *boff = nullptr;
       uint32_t k = 32, b0 = 0, nb = 0;
@@ -890,7 +986,8 @@ uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *
         nb = (ue + k - 1) / k - b0;
       }
       if (nb) {
-        size_t smem = (size_t)CT_WARPS * warp_stride(cap, mode != 0) * sizeof(uint32_t);
+        const uint32_t rcap = fit_cap(cap, mode != 0);
+        size_t smem = (size_t)CT_WARPS * warp_stride(rcap, mode != 0) * sizeof(uint32_t);
         auto range_fn = mode == 2 ? count_range_kernel<2> : mode == 1 ? count_range_kernel<1> : count_range_kernel<0>;
         int occ = occupancy((const void *)range_fn, CT_THREADS, smem);
         unsigned grid = (unsigned)std::min<uint64_t>(nb, (uint64_t)num_sms() * occ);
@@ -899,7 +996,7 @@ uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *
         TC_CUDA(cudaMemsetAsync(bctr.get(), 0, sizeof(unsigned), s));
         if (kernel_ms) TC_CUDA(cudaEventRecord(e0, s));
         ProfScope prof("count_range", s, 0.0);
-        range_fn<<<grid, CT_THREADS, smem, s>>>(g.offs.get(), g.col.get(), boff, k, b0, nb, ub, ue, cap, bctr.get(),
+        range_fn<<<grid, CT_THREADS, smem, s>>>(g.offs.get(), g.col.get(), boff, k, b0, nb, ub, ue, rcap, bctr.get(),
                                                 dT.get(), tv);
         TC_LAUNCH_CHECK();
         if (kernel_ms) TC_CUDA(cudaEventRecord(e1, s));
@@ -932,6 +1029,7 @@ uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *
           cap_small = std::max<uint32_t>(32, std::min<uint32_t>(cap, 1u << (b + 1)));
           break;
         }
+      cap_small = fit_cap(cap_small, mode != 0);
       nlaunch += 2;
       if (nitems) {
         DevBuf<uint64_t> items;

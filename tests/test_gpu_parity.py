@@ -392,3 +392,29 @@ def test_sort_merge_intersection(sched, cap):
     finally:
         tc.tc_set_option("intersect", 0)
         tc.tc_set_option("small_cap", 256)
+
+
+# ---------------------------------------------------------------- bitmap intersection (Bisson, Fig.13)
+def test_bitmap_intersection():
+    """Option "intersect"=2 (Bisson's block-per-vertex bitmap pattern) counts the
+    oracle's T under every directing / ordering rule, with the bitmap in shared memory
+    (|V| <= 2^20) and in per-CTA global slices (|V| > 2^20: isolated padding vertices)."""
+    tc.tc_set_option("intersect", 2)
+    try:
+        for seed, (sc, ef) in enumerate(((12, 16), (13, 8))):
+            spec = graphgen.rmat_spec(sc, ef, 95 + seed)
+            src, dst = graphgen.generate_cpu(spec)
+            ref = oracle.run(src, dst, spec.n, "id", "none")
+            for N in (spec.n, (1 << 20) + 77):
+                for d, r in (("id", "none"), ("degree", "degree"), ("paper", "paper"), ("degree", "none")):
+                    g = tc.Graph(src, dst, N).direct(d).reorder(r)
+                    assert g.count() == ref["T"], (N, d, r)
+                    g.free()
+        for name in ("K12", "W9", "B10", "CP6", "petersen"):
+            edges, n, T, t = graphs.CLOSED_FORMS[name]
+            src, dst, N, perm = graphs.noisy_samples(edges, n, np.random.default_rng(4), pad=2)
+            g = tc.Graph(src, dst, N).direct("paper")
+            assert g.count() == T, name
+            g.free()
+    finally:
+        tc.tc_set_option("intersect", 0)

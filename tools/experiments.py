@@ -22,7 +22,7 @@ def main():
     ap.add_argument("--rules", default="id:none,degree:none,paper:none,degree:degree,degree:paper,paper:paper")
     ap.add_argument("--schedules", default="bucketed,range")
     ap.add_argument("--reps", type=int, default=3)
-    ap.add_argument("--intersect", default="0", help="comma list: 0 binary search, 1 sort-merge (§6.2)")
+    ap.add_argument("--intersect", default="0", help="comma list: 0 binary search, 1 sort-merge (§6.2), 2 bitmap (Bisson, Fig.13)")
     a = ap.parse_args()
     spec = graphgen.CONFIGS[a.config]
     src = torch.empty(spec.samples, dtype=torch.int32, device="cuda")
@@ -52,7 +52,7 @@ def main():
             med = {k: statistics.median(x[k] for x in rows) for k in ("ms_build", "ms_direct", "ms_reorder", "ms_count")}
             tot = sum(med.values())
             m = st["m"]
-            print(f"| {d} | {r} | {sched} | {'sort-merge' if isect == '1' else 'binary search'} | {med['ms_build']:.2f} | {med['ms_direct']:.2f} | {med['ms_reorder']:.2f} | "
+            print(f"| {d} | {r} | {sched} | { {'0': 'binary search', '1': 'sort-merge', '2': 'bitmap'}[isect]} | {med['ms_build']:.2f} | {med['ms_direct']:.2f} | {med['ms_reorder']:.2f} | "
                   f"{med['ms_count']:.2f} | {tot:.2f} | {m / med['ms_count'] / 1e6:.2f} | {m / tot / 1e6:.2f} | "
                   f"{st['max_outdeg']} | {st['eq1']} | {st['eq3']} | {T} |", flush=True)
 
