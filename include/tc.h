@@ -186,7 +186,12 @@ tc_status tc_export_buckets(tc_graph *g, uint32_t *bucket_off);
  * tc_count / tc_count_range / tc_count_dist without per-vertex output), "peel_coop" (0/1:
  * run the whole A-direction peel as one cooperative launch with grid-wide barriers instead
  * of 5 launches and a host round trip per subround, default 1), "trim_memory" (any
- * value: release the library's cached device blocks). */
+ * value: release the library's cached device blocks), "extra_compute" (-1 = off, the
+ * default; q in 0..1024: counts run an instrumented copy of the warp-item kernel that
+ * performs p_c = q/8 extra searches of the staged N+(u) per wedge (whole 32-wedge warp
+ * steps, spread evenly), results discarded — the
+ * balance-point experiment of §5.3, used to re-fit the A-order model on B200
+ * (tools/refit.py); counts are unchanged). */
 tc_status tc_set_option(const char *key, int64_t value);
 
 /* Per-kernel profile since the last reset, as JSON text into buf (host, cap bytes):

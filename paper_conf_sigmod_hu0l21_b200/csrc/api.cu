@@ -183,6 +183,10 @@ tc_status tc_set_option(const char *key, int64_t value) {
     else if (k == "l2_persist") g_opt_l2_persist = value ? 1 : 0;
     else if (k == "trim_memory") dev_trim();
     else if (k == "bracket") g_opt_bracket = value ? 1 : 0;
+    else if (k == "extra_compute") {
+      TC_REQUIRE(value >= -1 && value <= 1024, ST_INVALID, "extra_compute: -1 (off) or 0..1024");
+      g_opt_extra = (int)value;
+    }
     else if (k == "intersect") {
       TC_REQUIRE(value >= 0 && value <= 2, ST_INVALID, "intersect: 0 = binary search, 1 = sort-merge, 2 = bitmap");
       g_opt_intersect = (int)value;

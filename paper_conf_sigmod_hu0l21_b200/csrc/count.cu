@@ -30,6 +30,7 @@ namespace tc {
 int g_opt_small_cap = 256;   // power of two: d~ below it -> warp items, else CTA items
 int g_opt_bracket = 1;       // bracketed binary search for long staged lists
 int g_opt_intersect = 0;     // 0 = binary search (the paper's kernel), 1 = sort-merge (P:548-550 comparison)
+int g_opt_extra = -1;        // §5.3 balance-point experiment: extra searches per wedge (-1 off)
 int g_opt_l2_persist = 0;    // L2 access-policy window over [offs | col] during counts (off: measured slower overall)
 
 namespace {
@@ -81,6 +82,8 @@ __host__ __device__ constexpr uint32_t warp_stride(uint32_t cap, bool pv) {
 
 __constant__ int g_bracket = 1;  // bracketed binary search on (option "bracket")
 __constant__ int g_merge = 0;    // sort-merge intersection instead of binary search (option "intersect")
+__constant__ int g_extra = 0;    // MODE 3: extra searches per 8 wedges (option "extra_compute", §5.3 p_c)
+__constant__ uint32_t g_sink_mask = 0;
 
 // Sort-merge intersection (the strategy the paper compares binary search against, §6.2,
 // P:548-550, Fig.10): lane l intersects N+(u) (`list`, ascending, shared or global) with
@@ -228,6 +231,16 @@ __device__ __forceinline__ void wedge_block(uint32_t j0, uint32_t last, const ui
     uint32_t pos;
     const bool hit = search(w[k], pos) && j0 + 32 * k <= last;
     cnt += hit ? 1u : 0u;
+    if (MODE == 3) {  // the paper's balance-point experiment (§5.3): p_c extra
+      uint32_t acc = 0;  // searches of the staged list per wedge (g_extra in 1/8 units), results kept alive
+      const uint32_t wi = (j0 >> 5) + k;  // 32-wedge step index: warp-uniform extra work
+      const int ne = (int)((((uint64_t)wi + 1) * (uint32_t)g_extra) >> 3) - (int)(((uint64_t)wi * (uint32_t)g_extra) >> 3);
+      for (int e = 0; e < ne; ++e) {
+        uint32_t p2;
+        acc += search(w[k] ^ (uint32_t)(e + 1), p2) ? 1u : 0u;
+      }
+      cnt += acc & g_sink_mask;  // 0 at run time, unknown to the compiler: keeps the searches
+    }
     if ((PV || PE) && hit) {
       atomicAdd(&ws.vcnt[ow[k]], 1u);
       if (cbase != 0xffffffffu) atomicAdd(&tc_smem[cbase + (pos - sbase)], 1u);
@@ -497,13 +510,13 @@ __global__ __launch_bounds__(256) void items_scatter_kernel(const uint64_t *__re
 // --------------------------------------------------------------- count kernels (a9)
 // Warp items; items [0, nheavy) are fetched one at a time, the rest CHUNK at a time.
 template <int MODE>
-__global__ __launch_bounds__(CT_THREADS, MODE == 0 ? 6 : 4) void count_small_kernel(const uint64_t *__restrict__ offs,
+__global__ __launch_bounds__(CT_THREADS, (MODE == 0 || MODE == 3) ? 6 : 4) void count_small_kernel(const uint64_t *__restrict__ offs,
                                                                  const uint32_t *__restrict__ col,
                                                                  const uint64_t *__restrict__ items, uint64_t nitems,
                                                                  uint64_t nheavy, unsigned long long *ctr, uint32_t cap,
                                                                  unsigned long long *T, unsigned long long *tv) {
   __shared__ WarpScratch s_ws[CT_WARPS];
-  const uint32_t slice = warp_id() * warp_stride(cap, MODE != 0);
+  const uint32_t slice = warp_id() * warp_stride(cap, MODE == 1 || MODE == 2);
   WarpScratch &ws = s_ws[warp_id()];
   uint64_t acc = 0;
   while (true) {  // heavy items, one per fetch
@@ -666,7 +679,7 @@ __global__ __launch_bounds__(CT_THREADS) void count_range_kernel(const uint64_t 
                                                                  unsigned long long *T, unsigned long long *tv) {
   __shared__ WarpScratch s_ws[CT_WARPS];
   __shared__ uint32_t s_bucket;
-  const uint32_t slice = warp_id() * warp_stride(cap, MODE != 0);
+  const uint32_t slice = warp_id() * warp_stride(cap, MODE == 1 || MODE == 2);
   WarpScratch &ws = s_ws[warp_id()];
   uint64_t acc = 0;
   while (true) {  // buckets fetched dynamically: a CTA takes the next bucket when done
@@ -845,7 +858,7 @@ static void configure_kernels() {
   for (auto fn : {count_large_kernel<0>, count_large_kernel<1>, count_large_kernel<2>})
     TC_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)large_smem));
   int small_max = 200 * 1024;
-  for (auto fn : {count_small_kernel<0>, count_small_kernel<1>, count_small_kernel<2>})
+  for (auto fn : {count_small_kernel<0>, count_small_kernel<1>, count_small_kernel<2>, count_small_kernel<3>})
     TC_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, small_max));
   for (auto fn : {count_range_kernel<0>, count_range_kernel<1>, count_range_kernel<2>})
     TC_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, small_max));
@@ -910,11 +923,18 @@ static int occupancy(const void *fn, int threads, size_t smem) {
 
 uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *kernel_ms, uint64_t *launches,
                      int mode) {
-  if (mode < 0) mode = d_tv ? 1 : 0;  // 0 count, 1 per-vertex (t[n], new labels), 2 per-edge (CSR positions)
+  // 0 count, 1 per-vertex (t[n], new labels), 2 per-edge (CSR positions), 3 count with
+  // g_opt_extra extra searches per wedge in the warp-item kernel (§5.3 experiment)
+  if (mode < 0) mode = d_tv ? 1 : (g_opt_extra >= 0 ? 3 : 0);
+  const bool pv = mode == 1 || mode == 2;
   cudaStream_t s = g.stream;
   configure_kernels();
   {
-    static int last_bracket = 1, last_intersect = 0;
+    static int last_bracket = 1, last_intersect = 0, last_extra = -1;
+    if (g_opt_extra != last_extra && g_opt_extra >= 0) {
+      TC_CUDA(cudaMemcpyToSymbol(g_extra, &g_opt_extra, sizeof(int)));
+      last_extra = g_opt_extra;
+    }
     if (g_opt_bracket != last_bracket) {
       TC_CUDA(cudaMemcpyToSymbol(g_bracket, &g_opt_bracket, sizeof(int)));
       last_bracket = g_opt_bracket;
@@ -942,7 +962,7 @@ uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *
     TC_CUDA(cudaEventCreate(&e1));
   }
   L2Window l2win(s, g.csr_mem.get(), g.csr_mem.bytes());
-  if (ub < ue && g.m && mode == 0 && g_opt_intersect == 2) {
+  if (ub < ue && g.m && (mode == 0 || mode == 3) && g_opt_intersect == 2) {
     // bitmap intersection (Bisson's block-per-vertex pattern): its own schedule
     const bool in_smem = g.n <= BM_SMEM_MAX_N;
     const uint32_t words = (g.n + 31) / 32;
@@ -986,8 +1006,8 @@ uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *
         nb = (ue + k - 1) / k - b0;
       }
       if (nb) {
-        const uint32_t rcap = fit_cap(cap, mode != 0);
-        size_t smem = (size_t)CT_WARPS * warp_stride(rcap, mode != 0) * sizeof(uint32_t);
+        const uint32_t rcap = fit_cap(cap, pv);
+        size_t smem = (size_t)CT_WARPS * warp_stride(rcap, pv) * sizeof(uint32_t);
         auto range_fn = mode == 2 ? count_range_kernel<2> : mode == 1 ? count_range_kernel<1> : count_range_kernel<0>;
         int occ = occupancy((const void *)range_fn, CT_THREADS, smem);
         unsigned grid = (unsigned)std::min<uint64_t>(nb, (uint64_t)num_sms() * occ);
@@ -1029,7 +1049,7 @@ uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *
           cap_small = std::max<uint32_t>(32, std::min<uint32_t>(cap, 1u << (b + 1)));
           break;
         }
-      cap_small = fit_cap(cap_small, mode != 0);
+      cap_small = fit_cap(cap_small, pv);
       nlaunch += 2;
       if (nitems) {
         DevBuf<uint64_t> items;
@@ -1056,9 +1076,11 @@ uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *
         }
         uint64_t nsmall = nitems - nlarge;
         if (nsmall) {
-          size_t smem = (size_t)CT_WARPS * warp_stride(cap_small, mode != 0) * sizeof(uint32_t);
-          auto small_fn =
-              mode == 2 ? count_small_kernel<2> : mode == 1 ? count_small_kernel<1> : count_small_kernel<0>;
+          size_t smem = (size_t)CT_WARPS * warp_stride(cap_small, pv) * sizeof(uint32_t);
+          auto small_fn = mode == 3   ? count_small_kernel<3>
+                          : mode == 2 ? count_small_kernel<2>
+                          : mode == 1 ? count_small_kernel<1>
+                                      : count_small_kernel<0>;
           int occ = occupancy((const void *)small_fn, CT_THREADS, smem);
           uint64_t want = (nsmall + CT_WARPS - 1) / CT_WARPS;
           unsigned grid = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(want, (uint64_t)num_sms() * occ));
