@@ -63,7 +63,13 @@ typedef enum { TC_REORDER_NONE = 0, TC_REORDER_DEGREE = 1, TC_REORDER_PAPER = 2 
  * of bucket i — the block model A-order optimises ("every consecutive k vertices are
  * grouped into a bucket ... assigned to one block").  AUTO = BUCKETED (measured
  * faster on B200 for every ordering). */
-typedef enum { TC_SCHED_AUTO = 0, TC_SCHED_BUCKETED = 1, TC_SCHED_RANGE = 2 } tc_schedule;
+/* EDGE_AORDER: A-order with edge units (the paper's variant for per-edge schedules,
+ * P:638-640): the (u, 32-v chunk) work items of the bucketed schedule are the units, item
+ * superiority = sum over its edges u->v of S(d~(v)) (Q26), Algorithm 2 puts them
+ * in buckets of k items (tc_aorder_params of the last tc_reorder, else defaults), CTA i
+ * takes bucket i.  Built by tc_set_schedule when the oriented CSR exists (its device time
+ * added to ms_reorder), else by the first count after the CSR changes. */
+typedef enum { TC_SCHED_AUTO = 0, TC_SCHED_BUCKETED = 1, TC_SCHED_RANGE = 2, TC_SCHED_EDGE_AORDER = 3 } tc_schedule;
 
 /* A-order parameters (Alg.2 inputs "F_c, F_m, λ"; Eq.19-22).
  *   F_m(d) = BW(d)^alpha (Eq.19), F_c(d) = 1/d^beta (Eq.20); alpha = beta = 1/2 is
@@ -98,6 +104,8 @@ typedef struct {
   double ms_build, ms_direct, ms_reorder, ms_count; /* device time of the last call of each */
   double ms_count_kernel;        /* device time of the count kernels alone (last tc_count) */
   uint64_t count_launches;       /* kernels launched by the last tc_count */
+  int64_t eq3_units;             /* Eq.3 objective of the edge-unit buckets (EDGE_AORDER), else -1 */
+  uint64_t nunits;               /* edge units (active work items) in those buckets */
 } tc_stats_t;
 
 /* a1-a3.  Raw samples (src[i], dst[i]), i < num_edges; ids must be < num_vertices.
@@ -171,6 +179,11 @@ tc_status tc_export_graph(tc_graph *g, uint64_t *edges, uint32_t *degree);
 tc_status tc_export_direct(tc_graph *g, uint32_t *outdeg, uint32_t *sub, uint32_t *dsnap);
 /* A-order buckets: bucket_off[nbuckets+1] (host or device). */
 tc_status tc_export_buckets(tc_graph *g, uint32_t *bucket_off);
+/* Edge-unit A-order (TC_SCHED_EDGE_AORDER, built on demand): units[nunits] = the active
+ * work items in bucket order, each (u << 32) | c0 (source u in final labels, first v index
+ * c0 of its 32-edge chunk); unit_off[nbuckets_units+1] with nbuckets_units =
+ * ceil(nunits / k).  Host or device pointers. */
+tc_status tc_export_units(tc_graph *g, uint64_t *units, uint32_t *unit_off);
 
 /* Library options: "profile" (0/1: per-stage CUDA-event timing in tc_stats_t, default 1),
  * "kernel_profile" (0/1: per-kernel event pairs for tc_profile_report, default 0),

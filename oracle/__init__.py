@@ -62,6 +62,8 @@ def lib():
         L.orc_superiority.restype = i64
         L.orc_reorder_paper.argtypes = [u32, p, d, d, d, p, u32, u32, i32, p, p, p]
         L.orc_reorder_paper.restype = i32
+        L.orc_aorder_units.argtypes = [u32, p, p, u32, i32, p, p, p]
+        L.orc_aorder_units.restype = i32
         L.orc_objective_eq3.argtypes = [u32, p, p, p, d, d, d, p, u32]
         L.orc_objective_eq3.restype = i64
         L.orc_cost_eq1.argtypes = [u32, u64, p, p, p]
@@ -160,6 +162,56 @@ def reorder(od, rule, k=DEFAULT_K, lam=DEFAULT_LAMBDA, alpha=DEFAULT_ALPHA, beta
             raise ValueError("reorder_paper failed")
         return perm[:n], boff[: int(nb[0]) + 1].copy()
     raise ValueError(rule)
+
+
+def aorder_units(S, active, k=DEFAULT_K, order=0):
+    """Algorithm 2 over units with given superiorities (the edge-unit variant of
+    P:638-640): returns (pos[i] = new index of unit i, bucket_off)."""
+    S = np.ascontiguousarray(S, dtype=np.int64)
+    act = np.ascontiguousarray(active, dtype=np.uint8)
+    n = len(S)
+    pos = np.zeros(max(n, 1), dtype=np.uint32)
+    boff = np.zeros(n + 2, dtype=np.uint32)
+    nb = np.zeros(1, dtype=np.uint32)
+    if lib().orc_aorder_units(n, _p(S), _p(act), k, order, _p(pos), _p(boff), _p(nb)) != 0:
+        raise ValueError("aorder_units failed")
+    return pos[:n], boff[: int(nb[0]) + 1].copy()
+
+
+def edge_units(offs, col, k=DEFAULT_K, lam=DEFAULT_LAMBDA, alpha=DEFAULT_ALPHA, beta=DEFAULT_BETA,
+               bw=None, order=0):
+    """Edge-unit A-order (Q26): units are the per-edge schedule's work items
+    (u, c0) — 32 consecutive out-edges of u, u ascending, for d~(u) >= 2 — with superiority
+    the sum of S(d~(v)) over the item's edges u->v (0 for d~(v) = 0); a unit with no wedge
+    (every d~(v) = 0) takes no part.  Returns (units in bucket order as (u << 32) | c0,
+    bucket_off)."""
+    offs = np.asarray(offs, dtype=np.int64)
+    col = np.asarray(col)
+    od = np.diff(offs)
+    table = {}
+    items, sup, act = [], [], []
+    for u in range(len(od)):
+        d = int(od[u])
+        if d < 2:
+            continue
+        for c0 in range(0, d, 32):
+            s, a = 0, False
+            for v in col[offs[u] + c0: offs[u] + min(d, c0 + 32)]:
+                dv = int(od[v])
+                if dv:
+                    if dv not in table:
+                        table[dv] = superiority(dv, lam, alpha, beta, bw)
+                    s += table[dv]
+                    a = True
+            items.append((u << 32) | c0)
+            sup.append(s)
+            act.append(1 if a else 0)
+    pos, boff = aorder_units(np.array(sup, dtype=np.int64), np.array(act, dtype=np.uint8), k, order)
+    units = np.zeros(int(boff[-1]) if len(boff) else 0, dtype=np.uint64)
+    for i, it in enumerate(items):
+        if act[i]:
+            units[pos[i]] = it
+    return units, boff
 
 
 def oriented_csr(edges, n, dirs, perm):

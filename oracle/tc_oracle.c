@@ -41,6 +41,12 @@
  *                        neighbour).  pinned: Σ support = 3T, closed forms (K_n: n-2;
  *                        wheel: spokes 2, rim 1; book: spine k, pages 1; friendship: 1;
  *                        K_{a,b}: 0), brute force (A²∘A), t(v) = Σ_{e∋v} support(e) / 2.
+ *   orc_aorder_units     Algorithm 2 over arbitrary units with given superiorities (the
+ *                        vertex A-order calls it; the edge-unit variant of P:638-640 passes
+ *                        the per-edge schedule's work items, Q26).  pinned
+ *                        through orc_reorder_paper's pins, and directly: with all S equal
+ *                        it fills buckets round-robin; a unit-by-unit brute-force check
+ *                        of lines 6/12 (min / max mem_sup, smallest index) on random S.
  *   orc_cost_eq1         Eq.1 numerator Σ_u |n·d~(u) − m|, exact 128-bit
  *   orc_superiority      S(d) = llround(2^20 (F_m(d) − λ F_c(d))) (Eq.22; Q20)
  *   orc_objective_eq3    Eq.3 Σ_i |Σ_{v∈B_i} S(v)| with λ folded into S
@@ -362,18 +368,20 @@ static int cmp_lpt(const void *a, const void *b) {
   return (x > y) - (x < y);
 }
 
-int orc_reorder_paper(uint32_t n, const uint32_t *od, double lambda, double alpha, double beta,
-                      const double *bw, uint32_t bw_len, uint32_t k, int order, uint32_t *perm,
-                      uint32_t *bucket_off, uint32_t *nbuckets) {
+/* Algorithm 2 over n units with given superiorities S[i] (fixed point, λ folded in);
+ * unit i takes part iff active[i].  The vertex A-order below calls it with S(d~(v)) and
+ * active = (d~(v) > 0); the edge-unit variant (Q26) with the work
+ * items of the per-edge schedule.  Outputs pos[i] (new index; inactive units last, in
+ * unit order), bucket_off[b+1], *nbuckets = b. */
+int orc_aorder_units(uint32_t n, const int64_t *S, const uint8_t *active, uint32_t k, int order,
+                     uint32_t *perm, uint32_t *bucket_off, uint32_t *nbuckets) {
   if (k == 0) return -1;
   size_t nn = n ? n : 1;
-  int64_t *S = (int64_t *)calloc(nn, sizeof(int64_t));
   uint32_t *vmem = (uint32_t *)malloc(sizeof(uint32_t) * nn);
   uint32_t *vcomp = (uint32_t *)malloc(sizeof(uint32_t) * nn);
   uint32_t nmem = 0, ncomp = 0;
   for (uint32_t v = 0; v < n; ++v) {
-    if (od[v] == 0) continue;
-    S[v] = orc_superiority(od[v], lambda, alpha, beta, bw, bw_len);
+    if (!active[v]) continue;
     if (S[v] > 0) vmem[nmem++] = v;   /* line 3: memory dominated */
     else vcomp[ncomp++] = v;           /* line 4: computing dominated */
   }
@@ -419,12 +427,30 @@ int orc_reorder_paper(uint32_t n, const uint32_t *od, double lambda, double alph
       perm[members[(size_t)i * k + j]] = idx++;                 /* line 19-20 */
   }
   if (bucket_off) bucket_off[b] = idx;
-  for (uint32_t v = 0; v < n; ++v)                              /* Q16: d~ = 0 last */
-    if (od[v] == 0) perm[v] = idx++;
+  for (uint32_t v = 0; v < n; ++v)                              /* Q16: inactive last */
+    if (!active[v]) perm[v] = idx++;
   if (nbuckets) *nbuckets = b;
-  free(S); free(vmem); free(vcomp); free(mem_sup); free(cnt); free(members); free(q.h);
+  free(vmem); free(vcomp); free(mem_sup); free(cnt); free(members); free(q.h);
   free(rest);
   return 0;
+}
+
+int orc_reorder_paper(uint32_t n, const uint32_t *od, double lambda, double alpha, double beta,
+                      const double *bw, uint32_t bw_len, uint32_t k, int order, uint32_t *perm,
+                      uint32_t *bucket_off, uint32_t *nbuckets) {
+  if (k == 0) return -1;
+  size_t nn = n ? n : 1;
+  int64_t *S = (int64_t *)calloc(nn, sizeof(int64_t));
+  uint8_t *active = (uint8_t *)calloc(nn, 1);
+  for (uint32_t v = 0; v < n; ++v) {
+    if (od[v] == 0) continue;          /* Q16: d~ = 0 does no work, F_c(0) undefined */
+    S[v] = orc_superiority(od[v], lambda, alpha, beta, bw, bw_len);
+    active[v] = 1;
+  }
+  int r = orc_aorder_units(n, S, active, k, order, perm, bucket_off, nbuckets);
+  free(S);
+  free(active);
+  return r;
 }
 
 /* Eq.3 objective, with λ folded into S: Σ_i |Σ_{v∈B_i} S(v)| where bucket i

@@ -25,7 +25,7 @@ LIB_PATH = os.path.join(_HERE, "libtc_b200.so")
 TC_OK, TC_ERR_INVALID, TC_ERR_OOM, TC_ERR_CUDA, TC_ERR_NCCL, TC_ERR_STATE = range(6)
 DIRECT = {"id": 0, "degree": 1, "paper": 2}
 REORDER = {"none": 0, "degree": 1, "paper": 2}
-SCHEDULE = {"auto": 0, "bucketed": 1, "range": 2}
+SCHEDULE = {"auto": 0, "bucketed": 1, "range": 2, "edge_aorder": 3}
 _STATUS = {1: "TC_ERR_INVALID", 2: "TC_ERR_OOM", 3: "TC_ERR_CUDA", 4: "TC_ERR_NCCL", 5: "TC_ERR_STATE"}
 
 
@@ -50,7 +50,8 @@ class Stats(ctypes.Structure):
         ("triangles", ctypes.c_uint64), ("wedges", ctypes.c_uint64), ("alg_bytes", ctypes.c_uint64),
         ("ms_build", ctypes.c_double), ("ms_direct", ctypes.c_double),
         ("ms_reorder", ctypes.c_double), ("ms_count", ctypes.c_double),
-        ("ms_count_kernel", ctypes.c_double), ("count_launches", ctypes.c_uint64)]
+        ("ms_count_kernel", ctypes.c_double), ("count_launches", ctypes.c_uint64),
+        ("eq3_units", ctypes.c_int64), ("nunits", ctypes.c_uint64)]
 
     def as_dict(self):
         d = {f: getattr(self, f) for f, _ in self._fields_}
@@ -90,6 +91,7 @@ def lib():
             "tc_export_graph": [p, p, p],
             "tc_export_direct": [p, p, p, p],
             "tc_export_buckets": [p, p],
+            "tc_export_units": [p, p, p],
             "tc_set_option": [ctypes.c_char_p, i64],
             "tc_profile_report": [ctypes.c_char_p, u64, i32],
         }
@@ -256,6 +258,10 @@ def tc_export_buckets(g, bucket_off):
     _check(lib().tc_export_buckets(g, _ptr(bucket_off)))
 
 
+def tc_export_units(g, units, unit_off):
+    _check(lib().tc_export_units(g, _ptr(units), _ptr(unit_off)))
+
+
 def tc_profile_report(reset=True):
     import json
     buf = ctypes.create_string_buffer(1 << 16)
@@ -373,6 +379,17 @@ class Graph:
         b = np.zeros(nb + 1, dtype=np.uint32)
         tc_export_buckets(self._h, b)
         return b
+
+    def export_units(self, k=32):
+        """Edge-unit A-order (schedule "edge_aorder"): (units in bucket order, offsets)."""
+        # sized generously: units <= sum_u ceil(d~(u)/32) <= m, buckets = ceil(units / k)
+        m = self.stats()["m"]
+        u = np.zeros(max(m, 1), dtype=np.uint64)
+        off = np.zeros(max(m, 1) + 2, dtype=np.uint32)
+        tc_export_units(self._h, u, off)
+        nu = self.stats()["nunits"]
+        nb = (nu + k - 1) // k
+        return u[:nu], off[:nb + 1]
 
 
 def count_triangles(src, dst, num_vertices, direct="degree", reorder="none", per_vertex=False,

@@ -188,33 +188,23 @@ struct MonoQueue {
 };
 }  // namespace
 
-void aorder_host(const std::vector<uint32_t> &od, const tc_aorder_params &p, std::vector<uint32_t> &perm,
-                 std::vector<uint32_t> &bucket_off, int64_t &eq3) {
-  const size_t n = od.size();
-  const uint32_t k = p.k;
-  uint32_t maxd = 0;
-  for (uint32_t d : od) maxd = std::max(maxd, d);
-  // superiority per degree value (table when the degree range is modest)
-  std::vector<int64_t> table;
-  const bool use_table = maxd <= (1u << 24);
-  if (use_table) {
-    table.assign((size_t)maxd + 1, 0);
-    std::vector<uint8_t> seen((size_t)maxd + 1, 0);
-    for (uint32_t d : od) seen[d] = 1;
-    for (uint32_t d = 1; d <= maxd; ++d)
-      if (seen[d]) table[d] = memory_superiority(d, p);
-  }
-  auto S = [&](uint32_t d) -> int64_t { return use_table ? table[d] : memory_superiority(d, p); };
-
-  std::vector<uint32_t> vmem, vcomp;  // line 3-4, ascending id
+// Algorithm 2 over arbitrary units (vertices, or the edge units of the per-edge schedule,
+// P:638-640): unit i has superiority S[i] (fixed point, λ folded in) and takes part iff
+// active[i]; pos[i] = its new index (buckets in index order, members in insertion order;
+// inactive units last, in unit order); bucket_off[b+1]; eq3 = Eq.3 objective.
+void aorder_units(const std::vector<int64_t> &Sv, const std::vector<uint8_t> &active, uint32_t k, int order,
+                  std::vector<uint32_t> &perm, std::vector<uint32_t> &bucket_off, int64_t &eq3) {
+  const size_t n = Sv.size();
+  auto S = [&](uint32_t v) -> int64_t { return Sv[v]; };
+  std::vector<uint32_t> vmem, vcomp;  // line 3-4, ascending unit index
   for (size_t v = 0; v < n; ++v) {
-    if (od[v] == 0) continue;
-    if (S(od[v]) > 0) vmem.push_back((uint32_t)v);
+    if (!active[v]) continue;
+    if (S((uint32_t)v) > 0) vmem.push_back((uint32_t)v);
     else vcomp.push_back((uint32_t)v);
   }
-  if (p.order == 1) {  // LPT option (Q18): descending |S|, ties by id
+  if (order == 1) {  // LPT option (Q18): descending |S|, ties by index
     auto lpt = [&](uint32_t a, uint32_t b) {
-      int64_t x = std::llabs(S(od[a])), y = std::llabs(S(od[b]));
+      int64_t x = std::llabs(S(a)), y = std::llabs(S(b));
       return x != y ? x > y : a < b;
     };
     std::sort(vmem.begin(), vmem.end(), lpt);
@@ -230,12 +220,12 @@ void aorder_host(const std::vector<uint32_t> &od, const tc_aorder_params &p, std
   // index fit 63 bits (always for the default parameters), else the generic tree.
   int64_t smax = 0, smin1 = INT64_MAX, smin2 = INT64_MAX;  // max |S|; min nonzero |S| per phase
   for (uint32_t v : vmem) {
-    int64_t a = std::llabs(S(od[v]));
+    int64_t a = std::llabs(S(v));
     smax = std::max(smax, a);
     if (a) smin1 = std::min(smin1, a);
   }
   for (uint32_t v : vcomp) {
-    int64_t a = std::llabs(S(od[v]));
+    int64_t a = std::llabs(S(v));
     smax = std::max(smax, a);
     if (a) smin2 = std::min(smin2, a);
   }
@@ -249,7 +239,7 @@ void aorder_host(const std::vector<uint32_t> &od, const tc_aorder_params &p, std
       int64_t bk = q.top();                  // line 6
       bucket_of[v] = (uint32_t)bk;          // line 7
       fill[bk]++;
-      mem_sup[bk] += S(od[v]);               // line 8
+      mem_sup[bk] += S(v);               // line 8
       if (fill[bk] == k) alive[bk] = 0;
       q.update((size_t)bk, mem_sup[bk], alive[bk]);  // line 9
     }
@@ -259,7 +249,7 @@ void aorder_host(const std::vector<uint32_t> &od, const tc_aorder_params &p, std
       int64_t bk = q.top();                  // line 12
       bucket_of[v] = (uint32_t)bk;          // line 13
       fill[bk]++;
-      mem_sup[bk] += S(od[v]);               // line 14
+      mem_sup[bk] += S(v);               // line 14
       if (fill[bk] == k) alive[bk] = 0;
       q.update((size_t)bk, mem_sup[bk], alive[bk]);  // line 15
     }
@@ -281,7 +271,7 @@ void aorder_host(const std::vector<uint32_t> &od, const tc_aorder_params &p, std
         const size_t bk = (size_t)(q.top() & imask);  // line 6
         bucket_of[v] = (uint32_t)bk;        // line 7
         fill[bk]++;
-        mem_sup[bk] += S(od[v]);             // line 8
+        mem_sup[bk] += S(v);             // line 8
         if (fill[bk] == k) alive[bk] = 0;
         q.replace_top(pack(bk, mem_sup[bk], false), alive[bk]);  // line 9
       }
@@ -293,7 +283,7 @@ void aorder_host(const std::vector<uint32_t> &od, const tc_aorder_params &p, std
         const size_t bk = (size_t)(q.top() & imask);  // line 12
         bucket_of[v] = (uint32_t)bk;        // line 13
         fill[bk]++;
-        mem_sup[bk] += S(od[v]);             // line 14
+        mem_sup[bk] += S(v);             // line 14
         if (fill[bk] == k) alive[bk] = 0;
         q.replace_top(pack(bk, mem_sup[bk], true), alive[bk]);  // line 15
       }
@@ -318,7 +308,39 @@ void aorder_host(const std::vector<uint32_t> &od, const tc_aorder_params &p, std
   }
   uint32_t idx = bucket_off[b];
   for (size_t v = 0; v < n; ++v)
-    if (od[v] == 0) perm[v] = idx++;         // Q16
+    if (!active[v]) perm[v] = idx++;         // Q16
+}
+
+
+void aorder_host(const std::vector<uint32_t> &od, const tc_aorder_params &p, std::vector<uint32_t> &perm,
+                 std::vector<uint32_t> &bucket_off, int64_t &eq3) {
+  const size_t n = od.size();
+  uint32_t maxd = 0;
+  for (uint32_t d : od) maxd = std::max(maxd, d);
+  // superiority per degree value: a table over the degrees present when the range is modest
+  const bool use_table = maxd <= (1u << 24);
+  std::vector<int64_t> table;
+  if (use_table) {
+    table.assign((size_t)maxd + 1, 0);
+    std::vector<uint8_t> seen((size_t)maxd + 1, 0);
+    for (uint32_t d : od) seen[d] = 1;
+    for (uint32_t d = 1; d <= maxd; ++d)
+      if (seen[d]) table[d] = memory_superiority(d, p);
+  }
+  std::vector<int64_t> S(n, 0);
+  std::vector<uint8_t> active(n, 0);
+  for (size_t v = 0; v < n; ++v)
+    if (od[v]) {  // d~ = 0: no work, F_c(0) undefined (Q16)
+      S[v] = use_table ? table[od[v]] : memory_superiority(od[v], p);
+      active[v] = 1;
+    }
+  aorder_units(S, active, p.k, p.order, perm, bucket_off, eq3);
+}
+
+std::vector<int64_t> superiority_table(uint32_t maxd, const tc_aorder_params &p) {
+  std::vector<int64_t> table((size_t)maxd + 1, 0);
+  for (uint32_t d = 1; d <= maxd; ++d) table[d] = memory_superiority(d, p);
+  return table;
 }
 
 }  // namespace tc

@@ -272,6 +272,11 @@ tc_status tc_reorder(tc_graph *gp, tc_reorder_rule rule, const tc_aorder_params 
     Graph &g = checked(gp, G_DIRECTED);
     TC_REQUIRE(rule >= TC_REORDER_NONE && rule <= TC_REORDER_PAPER, ST_INVALID, "unknown reorder rule");
     tc_aorder_params prm = defaults_or(p);
+    // keep the parameters (bw copied) for the edge-unit schedule
+    g.abw.assign(prm.bw ? prm.bw : nullptr, prm.bw ? prm.bw + prm.bw_len : nullptr);
+    g.aparams = prm;
+    g.aparams.bw = g.abw.empty() ? nullptr : g.abw.data();
+    g.aparams_set = true;
     StageTimer t(g.stream);
     reorder_graph(g, rule, prm);
     g.ms_reorder = t.stop();
@@ -282,8 +287,16 @@ tc_status tc_reorder(tc_graph *gp, tc_reorder_rule rule, const tc_aorder_params 
 tc_status tc_set_schedule(tc_graph *gp, tc_schedule s) {
   return guard([&] {
     TC_REQUIRE(gp != nullptr, ST_INVALID, "graph is NULL");
-    TC_REQUIRE(s >= TC_SCHED_AUTO && s <= TC_SCHED_RANGE, ST_INVALID, "unknown schedule");
+    TC_REQUIRE(s >= TC_SCHED_AUTO && s <= TC_SCHED_EDGE_AORDER, ST_INVALID, "unknown schedule");
     gp->schedule = s;
+    if (s == TC_SCHED_EDGE_AORDER && gp->state >= G_DIRECTED && gp->csr_ready && !gp->units_ready) {
+      // the edge-unit A-order is preprocessing: built here (timed with the reorder stage)
+      // when the CSR exists, else lazily by the first count
+      TC_CUDA(cudaSetDevice(gp->device));
+      StageTimer t(gp->stream);
+      build_units(*gp);
+      gp->ms_reorder += t.stop();
+    }
   });
 }
 
@@ -491,6 +504,8 @@ tc_status tc_get_stats(const tc_graph *gp, tc_stats_t *o) {
     o->ms_count = g.ms_count;
     o->ms_count_kernel = g.ms_count_kernel;
     o->count_launches = g.count_launches;
+    o->eq3_units = g.units_ready ? g.eq3_units : -1;
+    o->nunits = g.units_ready && !g.h_unit_off.empty() ? g.h_unit_off.back() : 0;
   });
 }
 
@@ -553,6 +568,18 @@ tc_status tc_export_buckets(tc_graph *gp, uint32_t *bucket_off) {
     Graph &g = checked(gp, G_DIRECTED);
     TC_REQUIRE(!g.h_bucket_off.empty(), ST_STATE, "no A-order buckets (tc_reorder PAPER first)");
     copy_out(bucket_off, g.h_bucket_off.data(), 4ull * g.h_bucket_off.size(), g.stream);
+    TC_CUDA(cudaStreamSynchronize(g.stream));
+  });
+}
+
+tc_status tc_export_units(tc_graph *gp, uint64_t *units, uint32_t *unit_off) {
+  return guard([&] {
+    Graph &g = checked(gp, G_DIRECTED);
+    ensure_csr(g);
+    build_units(g);
+    const uint64_t nu = g.h_unit_off.back();
+    if (nu) copy_out(units, g.units.get(), 8ull * nu, g.stream);
+    copy_out(unit_off, g.h_unit_off.data(), 4ull * g.h_unit_off.size(), g.stream);
     TC_CUDA(cudaStreamSynchronize(g.stream));
   });
 }

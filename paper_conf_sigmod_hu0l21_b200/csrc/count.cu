@@ -768,6 +768,80 @@ __global__ __launch_bounds__(BM_THREADS) void count_bitmap_kernel(const uint64_t
   block_add_u64(acc, T);
 }
 
+// ---- edge-unit A-order (TC_SCHED_EDGE_AORDER)
+// Units = the (u, 32-v chunk) work items, u ascending, chunks ascending (d~(u) >= 2).
+// nitems[u] = ceil(d~(u) / 32) for d~(u) >= 2.
+__global__ void unit_count_kernel(const uint64_t *__restrict__ offs, uint32_t n, uint32_t *__restrict__ cnt) {
+  for (uint64_t u = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; u < n; u += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t d = (uint32_t)(offs[u + 1] - offs[u]);
+    cnt[u] = d >= 2 ? (d + SV - 1) / SV : 0u;
+  }
+}
+// Warp per source: item (u, c0) gets S = sum over its edges u->v of S(d~(v)) (table in
+// fixed point, 0 for d~(v) = 0) and active = some d~(v) >= 1 (it has wedges).
+__global__ void unit_sup_kernel(const uint64_t *__restrict__ offs, const uint32_t *__restrict__ col, uint32_t n,
+                                const uint64_t *__restrict__ ioff, const int64_t *__restrict__ stab,
+                                uint64_t *__restrict__ items, int64_t *__restrict__ isup,
+                                uint8_t *__restrict__ iact) {
+  const uint64_t nw = (uint64_t)gridDim.x * (blockDim.x / 32);
+  for (uint64_t u = (uint64_t)blockIdx.x * (blockDim.x / 32) + warp_id(); u < n; u += nw) {
+    const uint64_t a = offs[u];
+    const uint32_t d = (uint32_t)(offs[u + 1] - a);
+    if (d < 2) continue;
+    const uint64_t base = ioff[u];
+    for (uint32_t c = 0; c * SV < d; ++c) {
+      const uint32_t j = c * SV + lane_id();
+      int64_t sv = 0;
+      bool act = false;
+      if (j < d) {
+        const uint32_t v = col[a + j];
+        const uint32_t dv = (uint32_t)(offs[v + 1] - offs[v]);
+        if (dv) {
+          sv = stab[dv];
+          act = true;
+        }
+      }
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) sv += __shfl_xor_sync(0xffffffffu, sv, o);
+      const unsigned any = __ballot_sync(0xffffffffu, act);
+      if (lane_id() == 0) {
+        items[base + c] = (u << 32) | (uint64_t)(c * SV);
+        isup[base + c] = sv;
+        iact[base + c] = any ? 1 : 0;
+      }
+    }
+  }
+}
+// CTA per bucket of units (fetched dynamically); the bucket's items dealt to the warps.
+template <int MODE>
+__global__ __launch_bounds__(CT_THREADS) void count_units_kernel(const uint64_t *__restrict__ offs,
+                                                                 const uint32_t *__restrict__ col,
+                                                                 const uint64_t *__restrict__ units,
+                                                                 const uint32_t *__restrict__ uoff, uint32_t nb,
+                                                                 uint32_t ub, uint32_t ue, uint32_t cap,
+                                                                 unsigned *bucket_ctr, unsigned long long *T,
+                                                                 unsigned long long *tv) {
+  __shared__ WarpScratch s_ws[CT_WARPS];
+  __shared__ uint32_t s_bucket;
+  const uint32_t slice = warp_id() * warp_stride(cap, MODE == 1 || MODE == 2);
+  WarpScratch &ws = s_ws[warp_id()];
+  uint64_t acc = 0;
+  while (true) {
+    __syncthreads();
+    if (threadIdx.x == 0) s_bucket = atomicAdd(bucket_ctr, 1u);
+    __syncthreads();
+    const uint32_t bi = s_bucket;
+    if (bi >= nb) break;
+    for (uint32_t i = uoff[bi] + warp_id(); i < uoff[bi + 1]; i += CT_WARPS) {
+      const uint64_t it = units[i];
+      const uint32_t u = (uint32_t)(it >> 32);
+      if (u < ub || u >= ue) continue;  // tc_count_range / tc_count_dist slices
+      acc += warp_item<MODE>(offs, col, u, (uint32_t)it, slice, cap, ws, tv);
+    }
+  }
+  block_add_u64(acc, T);
+}
+
 __global__ void gather_tv_kernel(const unsigned long long *__restrict__ tnew, const uint32_t *__restrict__ perm,
                                  uint32_t n, uint64_t *__restrict__ out) {
   for (uint64_t v = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (uint64_t)gridDim.x * blockDim.x)
@@ -861,6 +935,8 @@ static void configure_kernels() {
   for (auto fn : {count_small_kernel<0>, count_small_kernel<1>, count_small_kernel<2>, count_small_kernel<3>})
     TC_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, small_max));
   for (auto fn : {count_range_kernel<0>, count_range_kernel<1>, count_range_kernel<2>})
+    TC_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, small_max));
+  for (auto fn : {count_units_kernel<0>, count_units_kernel<1>, count_units_kernel<2>})
     TC_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, small_max));
   TC_CUDA(cudaFuncSetAttribute(count_bitmap_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                (int)(BM_SMEM_MAX_N / 8)));
@@ -987,6 +1063,26 @@ uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *
     TC_LAUNCH_CHECK();
     if (kernel_ms) TC_CUDA(cudaEventRecord(e1, s));
     ++nlaunch;
+  } else if (ub < ue && g.m && sched == TC_SCHED_EDGE_AORDER) {
+    build_units(g);
+    const uint32_t nb = (uint32_t)g.h_unit_off.size() - 1;
+    if (nb) {
+      const uint32_t rcap = fit_cap(cap, pv);
+      size_t smem = (size_t)CT_WARPS * warp_stride(rcap, pv) * sizeof(uint32_t);
+      auto fn = mode == 2 ? count_units_kernel<2> : mode == 1 ? count_units_kernel<1> : count_units_kernel<0>;
+      int occ = occupancy((const void *)fn, CT_THREADS, smem);
+      unsigned grid = (unsigned)std::min<uint64_t>(nb, (uint64_t)num_sms() * occ);
+      DevBuf<unsigned> bctr;
+      bctr.alloc(1, s);
+      TC_CUDA(cudaMemsetAsync(bctr.get(), 0, sizeof(unsigned), s));
+      if (kernel_ms) TC_CUDA(cudaEventRecord(e0, s));
+      ProfScope prof("count_units", s, 0.0);
+      fn<<<grid, CT_THREADS, smem, s>>>(g.offs.get(), g.col.get(), g.units.get(), g.unit_off.get(), nb, ub, ue, rcap,
+                                        bctr.get(), dT.get(), tv);
+      TC_LAUNCH_CHECK();
+      if (kernel_ms) TC_CUDA(cudaEventRecord(e1, s));
+      ++nlaunch;
+    }
   } else if (ub < ue && g.m) {
     if (sched == TC_SCHED_RANGE) {
       const uint32_t *boff = nullptr;
@@ -1106,6 +1202,75 @@ uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *
   }
   if (launches) *launches = nlaunch;
   return hT;
+}
+
+// Edge-unit A-order: units and their superiority on the GPU, Algorithm 2 over the units on
+// the host (aorder_units, the same greedy as the vertex A-order), units uploaded in bucket
+// order.  Inactive units (no wedge) are dropped: they add nothing to T.
+void build_units(Graph &g) {
+  if (g.units_ready) return;
+  cudaStream_t s = g.stream;
+  const uint32_t n = g.n;
+  tc_aorder_params prm = g.aparams;
+  if (!g.aparams_set) {
+    prm.lambda = 9.682;
+    prm.alpha = prm.beta = 0.5;
+    prm.bw = nullptr;
+    prm.bw_len = 0;
+    prm.k = 32;
+    prm.order = 0;
+  }
+  DevBuf<uint32_t> cnt;
+  DevBuf<uint64_t> ioff;
+  cnt.alloc(n ? n : 1, s);
+  ioff.alloc((uint64_t)n + 1, s);
+  if (n) {
+    unit_count_kernel<<<grid_for(n, 256), 256, 0, s>>>(g.offs.get(), n, cnt.get());
+    TC_LAUNCH_CHECK();
+  }
+  scan_u32_to_u64(cnt.get(), ioff.get(), n, s);
+  uint64_t nitems = 0;
+  TC_CUDA(cudaMemcpyAsync(&nitems, ioff.get() + n, 8, cudaMemcpyDeviceToHost, s));
+  TC_CUDA(cudaStreamSynchronize(s));
+  // superiority per out-degree value (fixed point, λ folded in); max d~ is label-free
+  ensure_od(g);
+  const uint32_t maxd = g.max_outdeg;
+  std::vector<int64_t> htab = superiority_table(maxd, prm);
+  DevBuf<int64_t> stab;
+  stab.alloc(htab.size(), s);
+  TC_CUDA(cudaMemcpyAsync(stab.get(), htab.data(), 8 * htab.size(), cudaMemcpyHostToDevice, s));
+  DevBuf<uint64_t> items;
+  DevBuf<int64_t> isup;
+  DevBuf<uint8_t> iact;
+  items.alloc(nitems ? nitems : 1, s);
+  isup.alloc(nitems ? nitems : 1, s);
+  iact.alloc(nitems ? nitems : 1, s);
+  if (nitems) {
+    unit_sup_kernel<<<grid_for((uint64_t)n * 32, 256), 256, 0, s>>>(g.offs.get(), g.col.get(), n, ioff.get(), stab.get(),
+                                                                    items.get(), isup.get(), iact.get());
+    TC_LAUNCH_CHECK();
+  }
+  std::vector<uint64_t> h_items(nitems);
+  std::vector<int64_t> h_sup(nitems);
+  std::vector<uint8_t> h_act(nitems);
+  if (nitems) {
+    TC_CUDA(cudaMemcpyAsync(h_items.data(), items.get(), 8 * nitems, cudaMemcpyDeviceToHost, s));
+    TC_CUDA(cudaMemcpyAsync(h_sup.data(), isup.get(), 8 * nitems, cudaMemcpyDeviceToHost, s));
+    TC_CUDA(cudaMemcpyAsync(h_act.data(), iact.get(), nitems, cudaMemcpyDeviceToHost, s));
+  }
+  TC_CUDA(cudaStreamSynchronize(s));
+  std::vector<uint32_t> pos;
+  aorder_units(h_sup, h_act, prm.k, prm.order, pos, g.h_unit_off, g.eq3_units);
+  const uint64_t nact = g.h_unit_off.back();
+  std::vector<uint64_t> ordered(nact ? nact : 1);
+  for (uint64_t i = 0; i < nitems; ++i)
+    if (h_act[i]) ordered[pos[i]] = h_items[i];
+  g.units.alloc(nact ? nact : 1, s);
+  g.unit_off.alloc(g.h_unit_off.size(), s);
+  if (nact) TC_CUDA(cudaMemcpyAsync(g.units.get(), ordered.data(), 8 * nact, cudaMemcpyHostToDevice, s));
+  TC_CUDA(cudaMemcpyAsync(g.unit_off.get(), g.h_unit_off.data(), 4 * g.h_unit_off.size(), cudaMemcpyHostToDevice, s));
+  TC_CUDA(cudaStreamSynchronize(s));  // host vectors must outlive the copies
+  g.units_ready = true;
 }
 
 void map_edges_canonical(Graph &g, const uint64_t *d_te, uint64_t *d_out) {

@@ -61,6 +61,16 @@ struct Graph {
 
   // a8 schedule
   int schedule = TC_SCHED_AUTO;
+  // A-order parameters of the last tc_reorder (bw copied), used by the edge-unit schedule
+  tc_aorder_params aparams{};
+  std::vector<double> abw;
+  bool aparams_set = false;
+  // edge-unit A-order (TC_SCHED_EDGE_AORDER): active items in bucket order + offsets
+  bool units_ready = false;
+  DevBuf<uint64_t> units;
+  DevBuf<uint32_t> unit_off;
+  std::vector<uint32_t> h_unit_off;
+  int64_t eq3_units = -1;
 
   // results / stats
   uint64_t triangles = 0, wedges = 0, alg_bytes = 0;
@@ -81,6 +91,9 @@ void build_oriented_csr(Graph &g);
 // aorder.cpp (host, Algorithm 2)
 void aorder_host(const std::vector<uint32_t> &od, const tc_aorder_params &p, std::vector<uint32_t> &perm,
                  std::vector<uint32_t> &bucket_off, int64_t &eq3);
+void aorder_units(const std::vector<int64_t> &S, const std::vector<uint8_t> &active, uint32_t k, int order,
+                  std::vector<uint32_t> &pos, std::vector<uint32_t> &bucket_off, int64_t &eq3);
+std::vector<int64_t> superiority_table(uint32_t maxd, const tc_aorder_params &p);
 // count.cu
 uint64_t count_graph(Graph &g, uint32_t u_begin, uint32_t u_end, uint64_t *d_tv /*new labels or null*/,
                      float *kernel_ms, uint64_t *launches, int mode = -1 /*-1: 1 if d_tv else 0; 2 = per-edge*/);
@@ -89,6 +102,7 @@ void map_edges_canonical(Graph &g, const uint64_t *d_te, uint64_t *d_out);
 void gather_per_vertex(Graph &g, const uint64_t *d_tnew, uint64_t *d_out);
 void partition_graph(Graph &g, uint32_t world, uint32_t *bounds);
 void analyze_graph(Graph &g);
+void build_units(Graph &g);  // edge-unit A-order buckets (count.cu)
 
 // options (api.cu)
 extern int g_opt_profile;

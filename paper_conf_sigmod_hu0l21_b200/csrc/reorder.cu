@@ -167,6 +167,7 @@ static void build_csr_split(Graph &g) {
   offs_sum_kernel<<<grid_for((uint64_t)n + 1, 256), 256, 0, s>>>(LF, LR.get(), n);
   TC_LAUNCH_CHECK();
   g.csr_ready = true;
+  g.units_ready = false;
 }
 
 void build_oriented_csr(Graph &g) {
@@ -214,6 +215,7 @@ void build_oriented_csr(Graph &g) {
     TC_CUDA(cudaMemsetAsync(g.offs.get(), 0, g.offs.bytes(), s));
   }
   g.csr_ready = true;
+  g.units_ready = false;
 }
 
 void reorder_graph(Graph &g, int rule, const tc_aorder_params &p) {

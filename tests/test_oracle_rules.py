@@ -221,3 +221,77 @@ def test_reorder_preserves_orientation():
             for v in base["col"][base["offs"][u]:base["offs"][u + 1]].tolist():
                 want.add((int(p[u]), int(p[v])))
         assert got == want
+
+
+# ---------------------------------------------------------------- Algorithm 2 over units (f3)
+def _greedy_scan(S, active, k, order=0):
+    """Algorithm 2 by exhaustive scan (no priority queue): line 6 takes the non-full bucket
+    of least (mem_sup, index), line 12 the non-full bucket of greatest mem_sup, ties by the
+    smallest index (P:424-438 with readings Q17-Q21)."""
+    idx = [i for i in range(len(S)) if active[i]]
+    mem = [i for i in idx if S[i] > 0]
+    comp = [i for i in idx if S[i] <= 0]
+    if order == 1:
+        key = lambda i: (-abs(int(S[i])), i)
+        mem.sort(key=key)
+        comp.sort(key=key)
+    b = (len(idx) + k - 1) // k
+    sup, members = [0] * b, [[] for _ in range(b)]
+    for v in mem:
+        bk = min((j for j in range(b) if len(members[j]) < k), key=lambda j: (sup[j], j))
+        members[bk].append(v)
+        sup[bk] += int(S[v])
+    for v in comp:
+        bk = min((j for j in range(b) if len(members[j]) < k), key=lambda j: (-sup[j], j))
+        members[bk].append(v)
+        sup[bk] += int(S[v])
+    pos, p = {}, 0
+    for j in range(b):
+        for v in members[j]:
+            pos[v] = p
+            p += 1
+    for i in range(len(S)):
+        if not active[i]:
+            pos[i] = p
+            p += 1
+    return [pos[i] for i in range(len(S))]
+
+
+@pytest.mark.parametrize("seed", range(12))
+def test_aorder_units_vs_exhaustive_scan(seed):
+    rng = np.random.default_rng(700 + seed)
+    n = int(rng.integers(1, 200))
+    S = rng.integers(-50, 50, size=n) * int(rng.integers(1, 1 << 20))
+    S[rng.random(n) < 0.1] = 0
+    active = (rng.random(n) < 0.85).astype(np.uint8)
+    k = int(rng.integers(1, 9))
+    order = seed % 2
+    pos, boff = oracle.aorder_units(S, active, k, order)
+    assert list(pos) == _greedy_scan(S, active, k, order)
+    assert boff[-1] == int(active.sum()) and np.all(np.diff(boff.astype(np.int64)) <= k)
+
+
+def test_aorder_units_equal_superiority_round_robin():
+    # all S equal and positive: phase 1 always takes the least-index bucket among those with
+    # the fewest members, i.e. unit i -> bucket i mod b, insertion order i // b
+    for b, k in ((5, 4), (7, 3), (1, 6)):
+        n = b * k
+        pos, boff = oracle.aorder_units(np.full(n, 3 << 20), np.ones(n, np.uint8), k)
+        assert list(pos) == [(i % b) * k + i // b for i in range(n)]
+        assert list(boff) == [j * k for j in range(b + 1)]
+
+
+def test_edge_units_cover_every_wedge_item():
+    """Edge units of a CSR: every (u, 32-edge chunk) with a wedge appears once."""
+    src, dst = graphgen.generate_cpu(graphgen.rmat_spec(9, 8, 31))
+    res = oracle.run(src, dst, 1 << 9, "degree", "none")
+    offs, col = res["offs"].astype(np.int64), res["col"]
+    units, boff = oracle.edge_units(offs, col, k=4)
+    od = np.diff(offs)
+    want = set()
+    for u in range(len(od)):
+        for c0 in range(0, int(od[u]) if od[u] >= 2 else 0, 32):
+            if (od[col[offs[u] + c0: offs[u] + min(od[u], c0 + 32)]] > 0).any():
+                want.add((u << 32) | c0)
+    assert sorted(units.tolist()) == sorted(want) and len(units) == len(want)
+    assert boff[-1] == len(units)
