@@ -40,6 +40,7 @@ constexpr int CT_WARPS = CT_THREADS / 32;
 constexpr int LG_THREADS = 256;       // large kernel: 8 warps
 constexpr int LG_WARPS = LG_THREADS / 32;
 constexpr uint32_t PIECE = 4096;      // large kernel: N+(u) piece in shared memory (16 KB)
+constexpr uint32_t LG_SUB = 16;       // large kernel: v's per dynamically fetched sub-chunk
 // bracket tables get 2^TS_* buckets per list element (finer buckets: fewer search steps)
 constexpr int TS_W = 2;               // warp items
 constexpr int TS_L = 1;               // CTA items (pieces)
@@ -584,6 +585,7 @@ __global__ __launch_bounds__(LG_THREADS, 5) void count_large_kernel(const uint64
   __shared__ uint32_t s_red[LG_WARPS];
   __shared__ __align__(8) uint64_t s_bar;
   __shared__ unsigned long long s_item;
+  __shared__ uint32_t s_next;  // next sub-chunk of the current piece
   WarpScratch &ws = s_ws[warp_id()];
   if (threadIdx.x == 0) mbar_init(&s_bar, 1);
   __syncthreads();
@@ -615,6 +617,7 @@ __global__ __launch_bounds__(LG_THREADS, 5) void count_large_kernel(const uint64
         tma_bulk_g2s(s_piece, col + abeg, bytes, &s_bar);
       }
       mbar_wait(&s_bar, phase);
+      if (threadIdx.x == 0) s_next = 0;  // published by the barrier below
       phase ^= 1u;
       const uint32_t *list = s_piece + shift;
       {  // pad the piece with +inf up to a power of two (+64) for the fixed-depth search
@@ -651,9 +654,16 @@ __global__ __launch_bounds__(LG_THREADS, 5) void count_large_kernel(const uint64
         __syncthreads();
       }
       uint32_t cnt = 0;
-      for (uint32_t c0 = cbeg + warp_id() * 32; c0 < cend; c0 += LG_THREADS) {
-        bool valid = c0 + lane_id() < cend;
-        uint32_t v = valid ? ldg_u32(col + a + c0 + lane_id()) : 0u;
+      // the item's v's in sub-chunks of LG_SUB fetched dynamically by the warps: the
+      // wedges behind each v vary widely, and a static 32-v share per warp left warps
+      // waiting at the end-of-piece barrier
+      while (true) {
+        uint32_t sc = 0;
+        if (lane_id() == 0) sc = atomicAdd(&s_next, 1u);
+        const uint32_t c0 = cbeg + __shfl_sync(0xffffffffu, sc, 0) * LG_SUB;
+        if (c0 >= cend) break;
+        const bool valid = lane_id() < LG_SUB && c0 + lane_id() < cend;
+        const uint32_t v = valid ? ldg_u32(col + a + c0 + lane_id()) : 0u;
         cnt += warp_chunk<MODE>(offs, col, v, valid, list, shift, S2 >= 0 ? tbase_lg : 0xffffffffu, 0xffffffffu, plen,
                                 true, lo, hi, ws, tv, c0 + lane_id(), a, a + p0, S2 >= 0 ? S2 : -2, sh);
       }
