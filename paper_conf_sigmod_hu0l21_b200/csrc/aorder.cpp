@@ -119,14 +119,16 @@ struct MonoQueue {
   int shift = 0;
   uint64_t bin0 = 0;
   std::vector<std::vector<uint64_t>> bins;
+  // the current (lowest non-empty) bin, sorted once when it becomes current: it is then
+  // consumed in order; keys re-inserted into the current bin (increments smaller than the
+  // bin width) go to a small heap beside it.  Exact: the queue pops the same strictly
+  // increasing sequence of unique packed keys as a single heap would.
+  std::vector<uint64_t> run, tmp;
+  size_t rpos = 0;
   std::vector<uint64_t> heap;
   size_t cur = 0;
   size_t bin_of(uint64_t pk) const { return (size_t)((pk >> shift) - bin0); }
-  // 4-ary min-heap: the children of i are 4i+1 .. 4i+4 (32 B), the smallest found
-  // branch-free; at the water level of phase 2 thousands of buckets share a bin, and the
-  // 4-ary layout halves the levels and the mispredicted branches of a binary heap
-  // (measured: 4-ary ~12% faster than binary and than 8-ary on a 16.7M-vertex A-order).
-  static constexpr size_t D = 4;
+  static constexpr size_t D = 4;  // 4-ary min-heap, children 4i+1 .. 4i+4
   void sift_down(size_t i) {
     const size_t n = heap.size();
     uint64_t *h = heap.data();
@@ -136,41 +138,61 @@ struct MonoQueue {
       if (c >= n) break;
       size_t best = c;
       uint64_t bv = h[c];
-      if (c + D <= n) {
-#pragma GCC unroll 4
-        for (size_t j = 1; j < D; ++j) {
-          const uint64_t v = h[c + j];
-          const bool lt = v < bv;
-          bv = lt ? v : bv;
-          best = lt ? c + j : best;
+      for (size_t j = c + 1; j < n && j < c + D; ++j)
+        if (h[j] < bv) {
+          bv = h[j];
+          best = j;
         }
-      } else {
-        for (size_t j = c + 1; j < n; ++j)
-          if (h[j] < bv) {
-            bv = h[j];
-            best = j;
-          }
-      }
       if (bv >= x) break;
       h[i] = bv;
       i = best;
     }
     h[i] = x;
   }
-  void heapify() {
-    if (heap.size() > 1)
-      for (size_t i = (heap.size() - 2) / D + 1; i-- > 0;) sift_down(i);
+  void push(uint64_t x) {
+    heap.push_back(x);
+    size_t i = heap.size() - 1;
+    while (i > 0) {
+      const size_t p = (i - 1) / D;
+      if (heap[p] <= x) break;
+      heap[i] = heap[p];
+      i = p;
+    }
+    heap[i] = x;
+  }
+  // LSD radix sort of the current bin on its low `shift` bits (the high bits are the bin)
+  void sort_run() {
+    const size_t n = run.size();
+    if (n < 64) {
+      std::sort(run.begin(), run.end());
+      return;
+    }
+    tmp.resize(n);
+    uint32_t cnt[256];
+    for (int b = 0; b < shift; b += 8) {
+      std::fill(cnt, cnt + 256, 0u);
+      for (size_t i = 0; i < n; ++i) ++cnt[(run[i] >> b) & 255];
+      uint32_t acc = 0;
+      for (int d = 0; d < 256; ++d) {
+        const uint32_t c = cnt[d];
+        cnt[d] = acc;
+        acc += c;
+      }
+      for (size_t i = 0; i < n; ++i) tmp[cnt[(run[i] >> b) & 255]++] = run[i];
+      run.swap(tmp);
+    }
   }
   void refill() {
-    while (heap.empty() && cur + 1 < bins.size()) {
+    while (rpos == run.size() && heap.empty() && cur + 1 < bins.size()) {
       ++cur;
-      heap.swap(bins[cur]);
-      heapify();
+      run.clear();
+      run.swap(bins[cur]);
+      sort_run();
+      rpos = 0;
     }
   }
   // keys: packed keys of the alive buckets; max_pk: upper bound of any key ever inserted;
-  // step: smallest key increment (packed units).  Bins ~step/8 wide so that the buckets
-  // bunched at the "water level" of phase 2 spread over many small heaps (<= 2^16 bins).
+  // step: smallest key increment (packed units).  Bins ~step/8 wide (<= 2^16 bins).
   void build(const std::vector<uint64_t> &keys, uint64_t max_pk, uint64_t step) {
     uint64_t mn = UINT64_MAX;
     for (uint64_t k : keys) mn = std::min(mn, k);
@@ -182,23 +204,33 @@ struct MonoQueue {
     bins.assign(((max_pk >> shift) - bin0) + 2, {});
     for (uint64_t k : keys) bins[bin_of(k)].push_back(k);
     cur = 0;
-    heap.swap(bins[0]);
-    heapify();
+    heap.clear();
+    run.clear();
+    run.swap(bins[0]);
+    sort_run();
+    rpos = 0;
     refill();
   }
-  bool empty() const { return heap.empty(); }
-  uint64_t top() const { return heap[0]; }
+  bool empty() const { return rpos == run.size() && heap.empty(); }
+  uint64_t top() const {
+    const uint64_t a = rpos < run.size() ? run[rpos] : UINT64_MAX;
+    const uint64_t b = heap.empty() ? UINT64_MAX : heap[0];
+    return a < b ? a : b;
+  }
   // the top's key grew to `pk` (alive) or its bucket left the queue (!alive)
   void replace_top(uint64_t pk, bool alive) {
-    if (alive && bin_of(pk) == cur) {
-      heap[0] = pk;
-      sift_down(0);
-      return;
+    if (rpos < run.size() && (heap.empty() || run[rpos] < heap[0])) {
+      ++rpos;
+    } else {
+      heap[0] = heap.back();
+      heap.pop_back();
+      if (!heap.empty()) sift_down(0);
     }
-    heap[0] = heap.back();
-    heap.pop_back();
-    if (!heap.empty()) sift_down(0);
-    if (alive) bins[bin_of(pk)].push_back(pk);
+    if (alive) {
+      const size_t bi = bin_of(pk);
+      if (bi == cur) push(pk);
+      else bins[bi].push_back(pk);
+    }
     refill();
   }
 };
