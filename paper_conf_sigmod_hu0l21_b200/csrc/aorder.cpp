@@ -20,6 +20,7 @@
 #include <cmath>
 #include <cstdint>
 #include <stdexcept>
+#include <thread>
 #include <vector>
 
 #include "../../include/tc.h"
@@ -240,15 +241,55 @@ struct MonoQueue {
 // P:638-640): unit i has superiority S[i] (fixed point, λ folded in) and takes part iff
 // active[i]; pos[i] = its new index (buckets in index order, members in insertion order;
 // inactive units last, in unit order); bucket_off[b+1]; eq3 = Eq.3 objective.
+// The O(n) passes around the sequential greedy (classification, relabel) run on all host
+// cores: f(lo, hi, t) over T contiguous chunks of [0, n).
+template <class F>
+static void par_chunks(size_t n, unsigned T, F f) {
+  if (T <= 1) {
+    f((size_t)0, n, 0u);
+    return;
+  }
+  std::vector<std::thread> th;
+  for (unsigned t = 0; t < T; ++t) th.emplace_back([&, t] { f(n * t / T, n * (t + 1) / T, t); });
+  for (auto &x : th) x.join();
+}
+static unsigned host_threads(size_t n) {
+  if (n < (1u << 20)) return 1;
+  unsigned h = std::thread::hardware_concurrency();
+  return std::max(1u, std::min(h ? h : 1u, 32u));
+}
+
 template <class SF, class AF>
 static void aorder_core(size_t n, SF S, AF active, uint32_t k, int order, std::vector<uint32_t> &perm,
                         std::vector<uint32_t> &bucket_off, int64_t &eq3) {
-  std::vector<uint32_t> vmem, vcomp;  // line 3-4, ascending unit index
-  for (size_t v = 0; v < n; ++v) {
-    if (!active(v)) continue;
-    if (S((uint32_t)v) > 0) vmem.push_back((uint32_t)v);
-    else vcomp.push_back((uint32_t)v);
+  // line 3-4: V_mem / V_comp in ascending unit index (per-chunk counts, then placement)
+  const unsigned T = host_threads(n);
+  std::vector<size_t> cm(T + 1, 0), cc(T + 1, 0), ci(T + 1, 0);
+  par_chunks(n, T, [&](size_t lo, size_t hi, unsigned t) {
+    size_t a = 0, c = 0, z = 0;
+    for (size_t v = lo; v < hi; ++v) {
+      if (!active(v)) ++z;
+      else if (S(v) > 0) ++a;
+      else ++c;
+    }
+    cm[t + 1] = a;
+    cc[t + 1] = c;
+    ci[t + 1] = z;
+  });
+  for (unsigned t = 0; t < T; ++t) {
+    cm[t + 1] += cm[t];
+    cc[t + 1] += cc[t];
+    ci[t + 1] += ci[t];
   }
+  std::vector<uint32_t> vmem(cm[T]), vcomp(cc[T]);
+  par_chunks(n, T, [&](size_t lo, size_t hi, unsigned t) {
+    size_t a = cm[t], c = cc[t];
+    for (size_t v = lo; v < hi; ++v) {
+      if (!active(v)) continue;
+      if (S(v) > 0) vmem[a++] = (uint32_t)v;
+      else vcomp[c++] = (uint32_t)v;
+    }
+  });
   if (order == 1) {  // LPT option (Q18): descending |S|, ties by index
     auto lpt = [&](uint32_t a, uint32_t b) {
       int64_t x = std::llabs(S(a)), y = std::llabs(S(b));
@@ -261,7 +302,7 @@ static void aorder_core(size_t n, SF S, AF active, uint32_t k, int order, std::v
   const size_t b = (nact + k - 1) / k;
   std::vector<int64_t> mem_sup(b, 0);        // line 1
   std::vector<uint32_t> fill(b, 0);
-  std::vector<uint32_t> bucket_of(n);  // insertion record, written in iteration order
+  std::vector<uint32_t> bucket_of(n), rank_of(n);  // insertion record: bucket, rank in it
   std::vector<uint8_t> alive(b, 1);
   // Phase 1 / phase 2 priority queues.  Packed 4-ary tree when max|mem_sup| and the bucket
   // index fit 63 bits (always for the default parameters), else the generic tree.
@@ -285,7 +326,7 @@ static void aorder_core(size_t n, SF S, AF active, uint32_t k, int order, std::v
     for (uint32_t v : vmem) {                // line 5
       int64_t bk = q.top();                  // line 6
       bucket_of[v] = (uint32_t)bk;          // line 7
-      fill[bk]++;
+      rank_of[v] = fill[bk]++;
       mem_sup[bk] += S(v);               // line 8
       if (fill[bk] == k) alive[bk] = 0;
       q.update((size_t)bk, mem_sup[bk], alive[bk]);  // line 9
@@ -295,7 +336,7 @@ static void aorder_core(size_t n, SF S, AF active, uint32_t k, int order, std::v
     for (uint32_t v : vcomp) {               // line 11
       int64_t bk = q.top();                  // line 12
       bucket_of[v] = (uint32_t)bk;          // line 13
-      fill[bk]++;
+      rank_of[v] = fill[bk]++;
       mem_sup[bk] += S(v);               // line 14
       if (fill[bk] == k) alive[bk] = 0;
       q.update((size_t)bk, mem_sup[bk], alive[bk]);  // line 15
@@ -317,7 +358,7 @@ static void aorder_core(size_t n, SF S, AF active, uint32_t k, int order, std::v
       for (uint32_t v : vmem) {              // line 5
         const size_t bk = (size_t)(q.top() & imask);  // line 6
         bucket_of[v] = (uint32_t)bk;        // line 7
-        fill[bk]++;
+        rank_of[v] = fill[bk]++;
         mem_sup[bk] += S(v);             // line 8
         if (fill[bk] == k) alive[bk] = 0;
         q.replace_top(pack(bk, mem_sup[bk], false), alive[bk]);  // line 9
@@ -329,7 +370,7 @@ static void aorder_core(size_t n, SF S, AF active, uint32_t k, int order, std::v
       for (uint32_t v : vcomp) {             // line 11
         const size_t bk = (size_t)(q.top() & imask);  // line 12
         bucket_of[v] = (uint32_t)bk;        // line 13
-        fill[bk]++;
+        rank_of[v] = fill[bk]++;
         mem_sup[bk] += S(v);             // line 14
         if (fill[bk] == k) alive[bk] = 0;
         q.replace_top(pack(bk, mem_sup[bk], true), alive[bk]);  // line 15
@@ -348,14 +389,12 @@ static void aorder_core(size_t n, SF S, AF active, uint32_t k, int order, std::v
     bucket_off[i + 1] = bucket_off[i] + fill[i];
     eq3 += std::llabs(mem_sup[i]);           // Eq.3 objective (λ folded into S)
   }
-  {
-    std::vector<uint32_t> cursor(bucket_off.begin(), bucket_off.end() - 1);
-    for (uint32_t v : vmem) perm[v] = cursor[bucket_of[v]]++;
-    for (uint32_t v : vcomp) perm[v] = cursor[bucket_of[v]]++;
-  }
-  uint32_t idx = bucket_off[b];
-  for (size_t v = 0; v < n; ++v)
-    if (!active(v)) perm[v] = idx++;         // Q16
+  // members in insertion order (bucket start + rank); inactive units last in unit order (Q16)
+  const uint32_t inactive0 = bucket_off[b];
+  par_chunks(n, T, [&](size_t lo, size_t hi, unsigned t) {
+    uint32_t idx = inactive0 + (uint32_t)ci[t];
+    for (size_t v = lo; v < hi; ++v) perm[v] = active(v) ? bucket_off[bucket_of[v]] + rank_of[v] : idx++;
+  });
 }
 
 
