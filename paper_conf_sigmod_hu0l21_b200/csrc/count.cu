@@ -40,7 +40,7 @@ constexpr int CT_WARPS = CT_THREADS / 32;
 constexpr int LG_THREADS = 256;       // large kernel: 8 warps
 constexpr int LG_WARPS = LG_THREADS / 32;
 constexpr uint32_t PIECE = 4096;      // large kernel: N+(u) piece in shared memory (16 KB)
-constexpr uint32_t LG_SUB = 16;       // large kernel: v's per dynamically fetched sub-chunk
+constexpr uint32_t LG_SUB = 8;        // large kernel: v's per dynamically fetched sub-chunk
 // bracket tables get 2^TS_* buckets per list element (finer buckets: fewer search steps)
 constexpr int TS_W = 2;               // warp items
 constexpr int TS_L = 1;               // CTA items (pieces)
@@ -438,12 +438,12 @@ __device__ __forceinline__ void block_add_u64(uint64_t v, unsigned long long *T)
 
 // --------------------------------------------------------------- schedule (a8)
 // Work items (u, c0): N+(u) is cut into chunks of SV = 32 v's (warp items, d~(u) < cap) or
-// LV = 512 v's (CTA items, d~(u) >= cap), so one heavy source never serialises on one
+// LV = 1024 v's (CTA items, d~(u) >= cap), so one heavy source never serialises on one
 // warp.  Items are grouped in floor(log2 d~(u)) bins, heaviest bin first (cf. the
 // logarithmic radix binning of P:63); within a bin the order is arbitrary (counts are
 // order-independent integers).
 constexpr uint32_t SV = 32;
-constexpr uint32_t LV = LG_THREADS;
+constexpr uint32_t LV = 1024;  // v's per CTA item (4 sub-chunk rounds per warp: fewer re-stagings of N+(u))
 
 __device__ __forceinline__ int deg_bin(uint32_t d) { return 31 - __clz(d); }  // floor(log2 d), d >= 1
 
