@@ -254,7 +254,7 @@ __device__ __forceinline__ void wedge_block(uint32_t j0, uint32_t last, const ui
 
 // All wedges of one chunk: blocks of 4 steps, then a 2- and a 1-step block for the rest
 // (an ER item has ~5 steps: 4 + 1 slots instead of 8).
-template <int MODE, class Search>
+template <int MODE, class Search, int NB = 4>
 __device__ __forceinline__ uint32_t wedge_loop(const uint32_t *__restrict__ col, const Search &search, uint32_t sbase,
                                                uint32_t cbase, uint32_t lo, uint32_t hi, uint32_t total,
                                                WarpScratch &ws, unsigned long long *tv, uint64_t ebase) {
@@ -263,6 +263,9 @@ __device__ __forceinline__ uint32_t wedge_loop(const uint32_t *__restrict__ col,
   const uint32_t *ob = col + ws.vb[0];  // element j of the current owner list is ob[j]
   const uint32_t last = total - 1, steps = (total + 31) >> 5, lane = lane_id();
   uint32_t st = 0;
+  if (NB == 8)  // CTA items (register budget 48): 8 gathers in flight per lane
+    for (; st + 8 <= steps; st += 8)
+      wedge_block<8, MODE>(lane + 32 * st, last, col, search, ws, o, o_end, ob, cnt, sbase, cbase, tv, ebase);
   for (; st + 4 <= steps; st += 4)
     wedge_block<4, MODE>(lane + 32 * st, last, col, search, ws, o, o_end, ob, cnt, sbase, cbase, tv, ebase);
   if (st + 2 <= steps) {
@@ -300,7 +303,7 @@ __device__ __forceinline__ int build_bracket(uint32_t sbase, uint32_t tbase, uin
 // lies in list[0..L) (w restricted to [lo, hi]).  `padded`: list is the shared-memory copy
 // tc_smem[sbase ..] padded with +inf to 2^ceil(log2 L) (+64) entries; tbase != ~0: room
 // for a bracket table.  Returns this lane's matches.
-template <int MODE>
+template <int MODE, int NB = 4>
 __device__ __forceinline__ uint32_t warp_chunk(const uint64_t *__restrict__ offs, const uint32_t *__restrict__ col,
                                                uint32_t v, bool valid, const uint32_t *list, uint32_t sbase,
                                                uint32_t tbase, uint32_t cbase, uint32_t L, bool padded, uint32_t lo,
@@ -342,7 +345,7 @@ __device__ __forceinline__ uint32_t warp_chunk(const uint64_t *__restrict__ offs
       switch (S2) {
 #define TC_TAB(k) \
   case k:                                                                                                     \
-    cnt = wedge_loop<MODE>(col, TabSearch<k>{smem_addr(sbase), smem_addr(tbase), lo, sh, ((hi - lo) >> sh) + 1, sbase}, \
+    cnt = wedge_loop<MODE, TabSearch<k>, NB>(col, TabSearch<k>{smem_addr(sbase), smem_addr(tbase), lo, sh, ((hi - lo) >> sh) + 1, sbase}, \
                            sbase, cbase, lo, hi, total, ws, tv, ebase);                                       \
     break;
         TC_TAB(0) TC_TAB(1) TC_TAB(2) TC_TAB(3) TC_TAB(4) TC_TAB(5) TC_TAB(6)
@@ -351,12 +354,12 @@ __device__ __forceinline__ uint32_t warp_chunk(const uint64_t *__restrict__ offs
     } else {
       switch (S) {
 #define TC_CASE(k) \
-  case k: cnt = wedge_loop<MODE>(col, Pow2Search<k>{smem_addr(sbase), sbase}, sbase, cbase, lo, hi, total, ws, tv, ebase); break;
+  case k: cnt = wedge_loop<MODE, Pow2Search<k>, NB>(col, Pow2Search<k>{smem_addr(sbase), sbase}, sbase, cbase, lo, hi, total, ws, tv, ebase); break;
         TC_CASE(1) TC_CASE(2) TC_CASE(3) TC_CASE(4) TC_CASE(5) TC_CASE(6) TC_CASE(7)
         TC_CASE(8) TC_CASE(9) TC_CASE(10) TC_CASE(11) TC_CASE(12) TC_CASE(13) TC_CASE(14)
 #undef TC_CASE
         default:
-          cnt = wedge_loop<MODE>(col, GlobalSearch{list, L, sbase}, sbase, 0xffffffffu, lo, hi, total, ws, tv, ebase);
+          cnt = wedge_loop<MODE, GlobalSearch, NB>(col, GlobalSearch{list, L, sbase}, sbase, 0xffffffffu, lo, hi, total, ws, tv, ebase);
       }
     }
   }
@@ -664,7 +667,7 @@ __global__ __launch_bounds__(LG_THREADS, 5) void count_large_kernel(const uint64
         if (c0 >= cend) break;
         const bool valid = lane_id() < LG_SUB && c0 + lane_id() < cend;
         const uint32_t v = valid ? ldg_u32(col + a + c0 + lane_id()) : 0u;
-        cnt += warp_chunk<MODE>(offs, col, v, valid, list, shift, S2 >= 0 ? tbase_lg : 0xffffffffu, 0xffffffffu, plen,
+        cnt += warp_chunk<MODE, MODE == 0 ? 8 : 4>(offs, col, v, valid, list, shift, S2 >= 0 ? tbase_lg : 0xffffffffu, 0xffffffffu, plen,
                                 true, lo, hi, ws, tv, c0 + lane_id(), a, a + p0, S2 >= 0 ? S2 : -2, sh);
       }
       ucnt += cnt;
