@@ -335,13 +335,20 @@ __device__ __forceinline__ uint32_t warp_chunk(const uint64_t *__restrict__ offs
     const int S = padded ? ceil_log2(L) : 0;
     int S2 = S2pre >= 0 ? S2pre : 99;  // S2pre: table prebuilt by the CTA (large kernel)
     uint32_t sh = shpre;
-    if (S2pre < 0 && S >= 6 && tbase != 0xffffffffu && g_bracket && total >= 2 * L) {
+    if (MODE != 4 && S2pre < 0 && S >= 6 && tbase != 0xffffffffu && g_bracket && total >= 2 * L) {
       const int span_bits = 32 - __clz(hi - lo);  // bits of (hi - lo)
       sh = span_bits > S + TS_W ? (uint32_t)(span_bits - S - TS_W) : 0u;
       S2 = build_bracket(sbase, tbase, L, lo, hi, sh);
       __syncwarp();
     }
-    if (S2 <= 6) {
+    if (MODE == 4) {  // every staged list has <= 32 entries (host-checked): 1..5 steps only
+      switch (S) {
+#define TC_SHORT(k) \
+  case k: cnt = wedge_loop<MODE, Pow2Search<k>, NB>(col, Pow2Search<k>{smem_addr(sbase), sbase}, sbase, cbase, lo, hi, total, ws, tv, ebase); break;
+        TC_SHORT(1) TC_SHORT(2) TC_SHORT(3) TC_SHORT(4) TC_SHORT(5)
+#undef TC_SHORT
+      }
+    } else if (S2 <= 6) {
       switch (S2) {
 #define TC_TAB(k) \
   case k:                                                                                                     \
@@ -514,7 +521,7 @@ __global__ __launch_bounds__(256) void items_scatter_kernel(const uint64_t *__re
 // --------------------------------------------------------------- count kernels (a9)
 // Warp items; items [0, nheavy) are fetched one at a time, the rest CHUNK at a time.
 template <int MODE>
-__global__ __launch_bounds__(CT_THREADS, (MODE == 0 || MODE == 3) ? 6 : 4) void count_small_kernel(const uint64_t *__restrict__ offs,
+__global__ __launch_bounds__(CT_THREADS, MODE == 4 ? 8 : (MODE == 0 || MODE == 3) ? 6 : 4) void count_small_kernel(const uint64_t *__restrict__ offs,
                                                                  const uint32_t *__restrict__ col,
                                                                  const uint64_t *__restrict__ items, uint64_t nitems,
                                                                  uint64_t nheavy, unsigned long long *ctr, uint32_t cap,
@@ -945,7 +952,8 @@ static void configure_kernels() {
   for (auto fn : {count_large_kernel<0>, count_large_kernel<1>, count_large_kernel<2>})
     TC_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)large_smem));
   int small_max = 200 * 1024;
-  for (auto fn : {count_small_kernel<0>, count_small_kernel<1>, count_small_kernel<2>, count_small_kernel<3>})
+  for (auto fn : {count_small_kernel<0>, count_small_kernel<1>, count_small_kernel<2>, count_small_kernel<3>,
+                  count_small_kernel<4>})
     TC_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, small_max));
   for (auto fn : {count_range_kernel<0>, count_range_kernel<1>, count_range_kernel<2>})
     TC_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, small_max));
@@ -1186,7 +1194,11 @@ uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *
         uint64_t nsmall = nitems - nlarge;
         if (nsmall) {
           size_t smem = (size_t)CT_WARPS * warp_stride(cap_small, pv) * sizeof(uint32_t);
-          auto small_fn = mode == 3   ? count_small_kernel<3>
+          // MODE 4: count with every warp-item list <= 32 entries (an ER graph): the
+          // short-list-only search dispatch needs 32 registers -> 8 CTAs (64 warps) per SM
+          const bool short_only = mode == 0 && cap_small == 32 && g_opt_intersect == 0;
+          auto small_fn = short_only  ? count_small_kernel<4>
+                          : mode == 3 ? count_small_kernel<3>
                           : mode == 2 ? count_small_kernel<2>
                           : mode == 1 ? count_small_kernel<1>
                                       : count_small_kernel<0>;
