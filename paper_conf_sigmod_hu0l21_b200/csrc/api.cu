@@ -183,6 +183,7 @@ tc_status tc_set_option(const char *key, int64_t value) {
     else if (k == "l2_persist") g_opt_l2_persist = value ? 1 : 0;
     else if (k == "trim_memory") dev_trim();
     else if (k == "bracket") g_opt_bracket = value ? 1 : 0;
+    else if (k == "lean") g_opt_lean = value ? 1 : 0;
     else if (k == "extra_compute") {
       TC_REQUIRE(value >= -1 && value <= 1024, ST_INVALID, "extra_compute: -1 (off) or 0..1024");
       g_opt_extra = (int)value;

@@ -30,6 +30,7 @@ namespace tc {
 int g_opt_small_cap = 256;   // power of two: d~ below it -> warp items, else CTA items
 int g_opt_bracket = 1;       // bracketed binary search for long staged lists
 int g_opt_intersect = 0;     // 0 = binary search (the paper's kernel), 1 = sort-merge (P:548-550 comparison)
+int g_opt_lean = 1;          // register-lean short-list count_small instantiation (MODE 4)
 int g_opt_extra = -1;        // §5.3 balance-point experiment: extra searches per wedge (-1 off)
 int g_opt_l2_persist = 0;    // L2 access-policy window over [offs | col] during counts (off: measured slower overall)
 
@@ -1196,7 +1197,9 @@ uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *
           size_t smem = (size_t)CT_WARPS * warp_stride(cap_small, pv) * sizeof(uint32_t);
           // MODE 4: count with every warp-item list <= 32 entries (an ER graph): the
           // short-list-only search dispatch needs 32 registers -> 8 CTAs (64 warps) per SM
-          const bool short_only = mode == 0 && cap_small == 32 && g_opt_intersect == 0;
+          // (a 32-register instantiation for lists <= 256 without the global path was
+          // measured 10% slower on R-MAT: issue-bound there, and it spills)
+          const bool short_only = g_opt_lean && mode == 0 && cap_small == 32 && g_opt_intersect == 0;
           auto small_fn = short_only  ? count_small_kernel<4>
                           : mode == 3 ? count_small_kernel<3>
                           : mode == 2 ? count_small_kernel<2>

@@ -109,6 +109,7 @@ extern int g_opt_profile;
 extern int g_opt_small_cap;
 extern int g_opt_l2_persist;
 extern int g_opt_bracket;
+extern int g_opt_lean;  // register-lean count_small instantiations
 extern int g_opt_extra;  // §5.3 experiment: extra searches per wedge (-1 = production kernel)
 extern int g_opt_intersect;  // 0 binary search, 1 sort-merge (count only)
 extern int g_opt_peel_coop;  // A-direction peel as one cooperative launch
