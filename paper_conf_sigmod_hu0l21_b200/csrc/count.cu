@@ -20,6 +20,9 @@
 //  * counts: u32 per lane per task, u64 per warp, block reduction, ONE 64-bit atomic per CTA.
 //  * per-vertex t(v): +1 at w and v per match (global atomics), warp total at u.
 #include <algorithm>
+#include <map>
+#include <mutex>
+#include <tuple>
 #include <vector>
 
 #include "internal.h"
@@ -1013,10 +1016,24 @@ static uint32_t fit_cap(uint32_t cap, bool pv) {
   return cap;
 }
 
+// Resident CTAs per SM, cached per (kernel, block, smem): queried on every count otherwise.
 static int occupancy(const void *fn, int threads, size_t smem) {
+  static std::mutex mu;
+  static std::map<std::tuple<const void *, int, size_t, int>, int> cache;
+  int dev = 0;
+  TC_CUDA(cudaGetDevice(&dev));
+  const auto key = std::make_tuple(fn, threads, smem, dev);
+  {
+    std::lock_guard<std::mutex> lk(mu);
+    auto it = cache.find(key);
+    if (it != cache.end()) return it->second;
+  }
   int blocks = 0;
   TC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&blocks, fn, threads, smem));
-  return blocks > 0 ? blocks : 1;
+  blocks = blocks > 0 ? blocks : 1;
+  std::lock_guard<std::mutex> lk(mu);
+  cache[key] = blocks;
+  return blocks;
 }
 
 uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *kernel_ms, uint64_t *launches,
@@ -1149,6 +1166,18 @@ uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *
       TC_LAUNCH_CHECK();
       bin_scan_kernel<<<1, 32, 0, s>>>(hist.get(), hist.get() + 32);
       TC_LAUNCH_CHECK();
+      // the item list is scattered before the host reads the bin sizes back (the scatter
+      // needs only the device-side cursors), into a buffer sized by the bound
+      // sum_u ceil(d~(u)/32) <= m/32 + #sources
+      DevBuf<uint64_t> items;
+      items.alloc(g.m / SV + (uint64_t)(ue - ub) + 1, s);
+      {
+        uint64_t span = 256ull * SC_PER_THREAD;
+        unsigned grid = (unsigned)std::min<uint64_t>((ue - ub + span - 1) / span, (uint64_t)num_sms() * 8);
+        items_scatter_kernel<<<grid, 256, 0, s>>>(g.offs.get(), ub, ue, cap, hist.get() + 32, items.get());
+        TC_LAUNCH_CHECK();
+        ++nlaunch;
+      }
       std::vector<unsigned long long> hh(32);
       TC_CUDA(cudaMemcpyAsync(hh.data(), hist.get(), 32 * sizeof(unsigned long long), cudaMemcpyDeviceToHost, s));
       TC_CUDA(cudaStreamSynchronize(s));
@@ -1170,15 +1199,6 @@ uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *
       cap_small = fit_cap(cap_small, pv);
       nlaunch += 2;
       if (nitems) {
-        DevBuf<uint64_t> items;
-        items.alloc(nitems, s);
-        {
-          uint64_t span = 256ull * SC_PER_THREAD;
-          unsigned grid = (unsigned)std::min<uint64_t>((ue - ub + span - 1) / span, (uint64_t)num_sms() * 8);
-          items_scatter_kernel<<<grid, 256, 0, s>>>(g.offs.get(), ub, ue, cap, hist.get() + 32, items.get());
-          TC_LAUNCH_CHECK();
-          ++nlaunch;
-        }
         if (kernel_ms) TC_CUDA(cudaEventRecord(e0, s));
         if (nlarge) {
           size_t smem = LG_SMEM_WORDS * sizeof(uint32_t);
