@@ -22,12 +22,24 @@ graphgen/libgraphgen.so: graphgen/graphgen_cpu.c graphgen/graphgen_cuda.cu graph
 	$(NVCC) $(ARCH) -shared graphgen/graphgen_cpu.o graphgen/graphgen_cuda.o -o $@ -lpthread
 
 oracle/liboracle.so: oracle/tc_oracle.c
-	$(CC) $(CFLAGS) -shared oracle/tc_oracle.c -o $@ -lm
+	$(CC) $(CFLAGS) -pthread -shared oracle/tc_oracle.c -o $@ -lm
 
-$(PKG)/libtc_b200.so: $(TC_SRCS) $(TC_HDRS) $(TC_CPP)
-	$(NVCC) $(NVFLAGS) -Iinclude -shared $(TC_SRCS) $(TC_CPP) -o $@ -ldl 2> $(PKG)/ptxas.log || (cat $(PKG)/ptxas.log; false)
+# one object per source (parallel make), then one shared library
+TC_OBJS := $(patsubst $(PKG)/csrc/%.cu,build/%.o,$(TC_SRCS)) $(patsubst $(PKG)/csrc/%.cpp,build/%.cpp.o,$(TC_CPP))
+
+build/%.o: $(PKG)/csrc/%.cu $(TC_HDRS) $(PKG)/csrc/internal.h
+	@mkdir -p build
+	$(NVCC) $(NVFLAGS) -Iinclude -c $< -o $@ 2> build/$*.ptxas.log || (cat build/$*.ptxas.log; false)
+
+build/%.cpp.o: $(PKG)/csrc/%.cpp $(TC_HDRS) $(PKG)/csrc/internal.h
+	@mkdir -p build
+	$(NVCC) $(NVFLAGS) -Iinclude -c $< -o $@
+
+$(PKG)/libtc_b200.so: $(TC_OBJS)
+	$(NVCC) $(ARCH) -shared $(TC_OBJS) -o $@ -ldl
+	cat build/*.ptxas.log > $(PKG)/ptxas.log
 
 clean:
-	rm -f graphgen/*.o graphgen/*.so oracle/*.so $(PKG)/*.so
+	rm -rf build graphgen/*.o graphgen/*.so oracle/*.so $(PKG)/*.so
 
 .PHONY: all clean

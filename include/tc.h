@@ -64,11 +64,13 @@ typedef enum { TC_REORDER_NONE = 0, TC_REORDER_DEGREE = 1, TC_REORDER_PAPER = 2 
  * grouped into a bucket ... assigned to one block").  AUTO = BUCKETED (measured
  * faster on B200 for every ordering). */
 /* EDGE_AORDER: A-order with edge units (the paper's variant for per-edge schedules,
- * P:638-640): the (u, 32-v chunk) work items of the bucketed schedule are the units, item
- * superiority = sum over its edges u->v of S(d~(v)) (Q26), Algorithm 2 puts them
- * in buckets of k items (tc_aorder_params of the last tc_reorder, else defaults), CTA i
- * takes bucket i.  Built by tc_set_schedule when the oriented CSR exists (its device time
- * added to ms_reorder), else by the first count after the CSR changes. */
+ * P:638-640 "edge is reorder unit ... resource usage tense of edges instead of vertices"):
+ * every directed edge u->v of the oriented CSR is a unit whose task streams N+(v) and
+ * binary-searches it in N+(u); its superiority is S(d~(v)) of the streamed list, d~(v) = 0
+ * -> no work, not a unit (Q26).  Algorithm 2 puts the units in buckets of k
+ * (tc_aorder_params of the last tc_reorder, else defaults), CTA i takes bucket i, a warp per
+ * unit.  Built by tc_set_schedule when the oriented CSR exists (its device time added to
+ * ms_reorder), else by the first count after the CSR changes. */
 typedef enum { TC_SCHED_AUTO = 0, TC_SCHED_BUCKETED = 1, TC_SCHED_RANGE = 2, TC_SCHED_EDGE_AORDER = 3 } tc_schedule;
 
 /* A-order parameters (Alg.2 inputs "F_c, F_m, λ"; Eq.19-22).
@@ -105,7 +107,8 @@ typedef struct {
   double ms_count_kernel;        /* device time of the count kernels alone (last tc_count) */
   uint64_t count_launches;       /* kernels launched by the last tc_count */
   int64_t eq3_units;             /* Eq.3 objective of the edge-unit buckets (EDGE_AORDER), else -1 */
-  uint64_t nunits;               /* edge units (active work items) in those buckets */
+  uint64_t nunits;               /* edge units (active edges) in those buckets */
+  uint64_t unit_buckets;         /* number of edge-unit buckets (EDGE_AORDER), else 0 */
 } tc_stats_t;
 
 /* a1-a3.  Raw samples (src[i], dst[i]), i < num_edges; ids must be < num_vertices.
@@ -125,6 +128,17 @@ tc_status tc_direct(tc_graph *g, tc_direct_rule rule);
 /* a6-a7.  p may be NULL (defaults above) and is ignored unless rule == PAPER.
  * Builds the oriented CSR in the new labels (lists ascending). */
 tc_status tc_reorder(tc_graph *g, tc_reorder_rule rule, const tc_aorder_params *p);
+
+/* a6-a7 on N ranks holding replicas of the same directed graph (a11 plumbing):
+ * identical result to tc_reorder on every rank, but for rule == PAPER the Algorithm 2
+ * greedy (sequential host work) runs on rank 0 only and pi / bucket_off / the Eq.3
+ * objective reach the other ranks by ncclBroadcast on the graph's stream (instead of N
+ * concurrent host greedies); other rules run locally.  nccl_comm: ncclComm_t from
+ * tc_nccl_comm_init, rank in [0, world).  Collective: every rank must call it.  Errors:
+ * TC_ERR_INVALID (bad comm/rank/world/params), TC_ERR_STATE (before tc_direct),
+ * TC_ERR_NCCL. */
+tc_status tc_reorder_dist(tc_graph *g, tc_reorder_rule rule, const tc_aorder_params *p, void *nccl_comm,
+                          int rank, int world);
 
 /* Schedule used by subsequent counts (TC_SCHED_AUTO by default). */
 tc_status tc_set_schedule(tc_graph *g, tc_schedule s);
@@ -180,9 +194,8 @@ tc_status tc_export_direct(tc_graph *g, uint32_t *outdeg, uint32_t *sub, uint32_
 /* A-order buckets: bucket_off[nbuckets+1] (host or device). */
 tc_status tc_export_buckets(tc_graph *g, uint32_t *bucket_off);
 /* Edge-unit A-order (TC_SCHED_EDGE_AORDER, built on demand): units[nunits] = the active
- * work items in bucket order, each (u << 32) | c0 (source u in final labels, first v index
- * c0 of its 32-edge chunk); unit_off[nbuckets_units+1] with nbuckets_units =
- * ceil(nunits / k).  Host or device pointers. */
+ * edge units in bucket order, each (u << 32) | j (source u in final labels, the edge
+ * u -> col[offs[u] + j]); unit_off[unit_buckets+1] (tc_stats_t).  Host or device pointers. */
 tc_status tc_export_units(tc_graph *g, uint64_t *units, uint32_t *unit_off);
 
 /* Library options: "profile" (0/1: per-stage CUDA-event timing in tc_stats_t, default 1),

@@ -49,11 +49,17 @@ def lib():
                                     ctypes.c_int64, ctypes.c_double, ctypes.c_void_p)
         L.orc_simple_graph.argtypes = [p, p, u64, u32, p]
         L.orc_simple_graph.restype = i64
+        L.orc_canonical_keys.argtypes = [p, p, u64, u32, p]
+        L.orc_canonical_keys.restype = i64
+        L.orc_unique_sorted.argtypes = [p, u64]
+        L.orc_unique_sorted.restype = u64
+        L.orc_oriented_keys.argtypes = [p, u64, p, p, p]
+        L.orc_csr_from_sorted_keys.argtypes = [p, u64, u32, p, p]
         L.orc_degrees.argtypes = [p, u64, u32, p]
         L.orc_sym_csr.argtypes = [p, u64, u32, p, p]
         L.orc_direct_id.argtypes = [u64, p]
         L.orc_direct_degree.argtypes = [p, u64, p, p]
-        L.orc_direct_paper.argtypes = [p, u64, u32, p, p, p, p, p, p, p]
+        L.orc_direct_paper.argtypes = [p, u64, u32, p, p, p, p, p, p]
         L.orc_direct_paper.restype = i32
         L.orc_outdeg.argtypes = [p, u64, u32, p, p]
         L.orc_reorder_none.argtypes = [u32, p]
@@ -67,9 +73,10 @@ def lib():
         L.orc_objective_eq3.argtypes = [u32, p, p, p, d, d, d, p, u32]
         L.orc_objective_eq3.restype = i64
         L.orc_cost_eq1.argtypes = [u32, u64, p, p, p]
-        L.orc_oriented_csr.argtypes = [p, u64, u32, p, p, p, p]
         L.orc_count_forward.argtypes = [u32, p, p, u32, u32, p]
         L.orc_count_forward.restype = u64
+        L.orc_count_forward_mt.argtypes = [u32, p, p, u32, u32, p, i32]
+        L.orc_count_forward_mt.restype = u64
         L.orc_local_triangles.argtypes = [p, p, u64, p, u32, u32, p]
         L.orc_local_triangles.restype = i32
         L.orc_edge_support.argtypes = [p, u64, p, p, p]
@@ -81,14 +88,17 @@ def lib():
 
 
 def simple_graph(src, dst, n):
-    """O1: sorted unique undirected edges as uint64 keys (min<<32 | max)."""
+    """O1: sorted unique undirected edges as uint64 keys (min<<32 | max).  The sort step is
+    numpy's (a library sort)."""
     src = np.ascontiguousarray(src, dtype=np.uint32)
     dst = np.ascontiguousarray(dst, dtype=np.uint32)
-    edges = np.empty(max(len(src), 1), dtype=np.uint64)
-    m = lib().orc_simple_graph(_p(src), _p(dst), len(src), n, _p(edges))
-    if m < 0:
+    keys = np.empty(max(len(src), 1), dtype=np.uint64)
+    k = lib().orc_canonical_keys(_p(src), _p(dst), len(src), n, _p(keys))
+    if k < 0:
         raise ValueError("vertex id >= n")
-    return edges[:m].copy()
+    keys[:k].sort()
+    m = lib().orc_unique_sorted(_p(keys), k)
+    return keys[:m]  # a view: no second M-sized buffer at full-size configs
 
 
 def degrees(edges, n):
@@ -115,13 +125,17 @@ def direct(edges, n, rule):
         deg = degrees(edges, n)
         lib().orc_direct_degree(_p(edges), m, _p(deg), _p(d))
     elif rule == "paper":
-        offs, adj = sym_csr(edges, n)
+        # list offsets of N(v): exclusive prefix sum of the degrees
+        offs = np.zeros(n + 1, dtype=np.uint64)
+        np.cumsum(degrees(edges, n), dtype=np.uint64, out=offs[1:])
         sub = np.zeros(max(n, 1), dtype=np.uint32)
         dsnap = np.zeros(max(n, 1), dtype=np.uint32)
         lv = np.zeros(1, dtype=np.uint32)
         sr = np.zeros(1, dtype=np.uint32)
-        lib().orc_direct_paper(_p(edges), m, n, _p(offs), _p(adj), _p(d), _p(sub), _p(dsnap),
-                               _p(lv), _p(sr))
+        if lib().orc_direct_paper(_p(edges), m, n, _p(offs), _p(d), _p(sub), _p(dsnap),
+                                  _p(lv), _p(sr)) != 0:
+            raise ValueError("orc_direct_paper: m >= 2^32 not supported")
+        del offs
         info = {"sub": sub[:n], "dsnap": dsnap[:n], "levels": int(lv[0]), "subrounds": int(sr[0])}
     else:
         raise ValueError(rule)
@@ -178,57 +192,71 @@ def aorder_units(S, active, k=DEFAULT_K, order=0):
     return pos[:n], boff[: int(nb[0]) + 1].copy()
 
 
+def edge_unit_superiority(offs, col, lam=DEFAULT_LAMBDA, alpha=DEFAULT_ALPHA, beta=DEFAULT_BETA,
+                          bw=None):
+    """Edge units (Q26): every directed edge u->v of the oriented CSR,
+    in CSR order, is a unit whose task streams N+(v) and binary-searches it in N+(u); its
+    superiority is that of the streamed list, S(d~(v)) (Eq.19-22 with the vertex model's
+    parameters); d~(v) = 0 means no work: not a unit (as Q16 for vertices).
+    Returns (S[m] int64, active[m] uint8), indexed by CSR position."""
+    offs = np.asarray(offs, dtype=np.int64)
+    od = np.diff(offs)
+    dv = od[np.asarray(col, dtype=np.int64)] if len(col) else np.zeros(0, np.int64)
+    table = {int(d): superiority(int(d), lam, alpha, beta, bw) for d in np.unique(dv) if d > 0}
+    S = np.array([table.get(int(d), 0) for d in dv], dtype=np.int64)
+    return S, (dv > 0).astype(np.uint8)
+
+
 def edge_units(offs, col, k=DEFAULT_K, lam=DEFAULT_LAMBDA, alpha=DEFAULT_ALPHA, beta=DEFAULT_BETA,
                bw=None, order=0):
-    """Edge-unit A-order (Q26): units are the per-edge schedule's work items
-    (u, c0) — 32 consecutive out-edges of u, u ascending, for d~(u) >= 2 — with superiority
-    the sum of S(d~(v)) over the item's edges u->v (0 for d~(v) = 0); a unit with no wedge
-    (every d~(v) = 0) takes no part.  Returns (units in bucket order as (u << 32) | c0,
-    bucket_off)."""
+    """Edge-unit A-order: Algorithm 2 (orc_aorder_units) over the edge units of
+    edge_unit_superiority.  Returns (units in bucket order as (u << 32) | j — the edge
+    u -> col[offs[u] + j] — and bucket_off)."""
     offs = np.asarray(offs, dtype=np.int64)
-    col = np.asarray(col)
-    od = np.diff(offs)
-    table = {}
-    items, sup, act = [], [], []
-    for u in range(len(od)):
-        d = int(od[u])
-        if d < 2:
-            continue
-        for c0 in range(0, d, 32):
-            s, a = 0, False
-            for v in col[offs[u] + c0: offs[u] + min(d, c0 + 32)]:
-                dv = int(od[v])
-                if dv:
-                    if dv not in table:
-                        table[dv] = superiority(dv, lam, alpha, beta, bw)
-                    s += table[dv]
-                    a = True
-            items.append((u << 32) | c0)
-            sup.append(s)
-            act.append(1 if a else 0)
-    pos, boff = aorder_units(np.array(sup, dtype=np.int64), np.array(act, dtype=np.uint8), k, order)
+    S, act = edge_unit_superiority(offs, col, lam, alpha, beta, bw)
+    pos, boff = aorder_units(S, act, k, order)
+    m = len(S)
+    src = np.repeat(np.arange(len(offs) - 1, dtype=np.int64), np.diff(offs))
+    j = np.arange(m, dtype=np.int64) - offs[src] if m else np.zeros(0, np.int64)
     units = np.zeros(int(boff[-1]) if len(boff) else 0, dtype=np.uint64)
-    for i, it in enumerate(items):
-        if act[i]:
-            units[pos[i]] = it
+    a = act.astype(bool)
+    units[pos[a].astype(np.int64)] = ((src[a] << 32) | j[a]).astype(np.uint64)
     return units, boff
 
 
 def oriented_csr(edges, n, dirs, perm):
+    """Oriented, relabelled CSR: the (pi(source), pi(target)) keys of the directed edges,
+    sorted (numpy's sort), counted into offsets."""
+    m = len(edges)
+    keys = np.empty(max(m, 1), dtype=np.uint64)
+    lib().orc_oriented_keys(_p(edges), m, _p(dirs), _p(np.ascontiguousarray(perm, dtype=np.uint32)),
+                            _p(keys))
+    keys[:m].sort()
     offs = np.zeros(n + 1, dtype=np.uint64)
-    col = np.zeros(max(len(edges), 1), dtype=np.uint32)
-    lib().orc_oriented_csr(_p(edges), len(edges), n, _p(dirs), _p(perm), _p(offs), _p(col))
-    return offs, col[: len(edges)]
+    col = np.zeros(max(m, 1), dtype=np.uint32)
+    lib().orc_csr_from_sorted_keys(_p(keys), m, n, _p(offs), _p(col))
+    del keys
+    return offs, col[:m]
 
 
-def count_forward(offs, col, u_begin=0, u_end=None, per_vertex=False):
+def count_forward(offs, col, u_begin=0, u_end=None, per_vertex=False, threads=1):
+    """O4 forward count over sources [u_begin, u_end); threads > 1 (or 0 = all online
+    cores) splits the sources over threads (orc_count_forward_mt)."""
     n = len(offs) - 1
     if u_end is None:
         u_end = n
     tv = np.zeros(max(n, 1), dtype=np.uint64) if per_vertex else None
     col = col if len(col) else np.zeros(1, dtype=np.uint32)
-    T = lib().orc_count_forward(n, _p(offs), _p(col), u_begin, u_end, _p(tv))
+    if threads == 1:
+        T = lib().orc_count_forward(n, _p(offs), _p(col), u_begin, u_end, _p(tv))
+    else:
+        T = lib().orc_count_forward_mt(n, _p(offs), _p(col), u_begin, u_end, _p(tv), threads)
     return (int(T), tv[:n]) if per_vertex else int(T)
+
+
+def host_cores():
+    """Threads orc_count_forward_mt uses with threads=0 (online cores)."""
+    return os.cpu_count() or 1
 
 
 def local_triangles(src, dst, vertices, max_deg=4096):

@@ -9,7 +9,8 @@
  * (taken from SURVEY.md §8(c)) where the paper is silent, ambiguous or garbled.
  *
  * What each function computes and what pins it (tests/test_oracle*.py):
- *   orc_simple_graph     O1  simple undirected graph (Q1)
+ *   orc_canonical_keys / O1  simple undirected graph (Q1): (min,max) keys,
+ *   orc_unique_sorted        sorted by a library sort (numpy), duplicates dropped
  *                            pinned: brute-force set semantics on random inputs
  *   orc_sym_csr          symmetric adjacency N(v), ascending ("nbrList")
  *   orc_direct_id        ID-based directing, u->v iff u<v (Q12)
@@ -27,7 +28,8 @@
  *                        readings Q15-Q21.  PARITY VS AUTHORS' CODE UNPINNED (Fig.8
  *                        BW curve not printed); pinned by: hand cases in
  *                        tests/golden/, bijection, bucket capacity, Eq.3 >= |sum S|.
- *   orc_oriented_csr     oriented + relabelled CSR, lists ascending
+ *   orc_oriented_keys /  oriented + relabelled CSR, lists ascending: (pi(s), pi(t)) keys,
+ *   orc_csr_from_sorted_keys    sorted by a library sort, then counted into offsets
  *   orc_count_forward    T = sum_u sum_{v in N+(u)} |N+(u) ∩ N+(v)| by two-pointer
  *                        merge (forward algorithm); per-vertex t(v).
  *                        pinned: closed forms (K_n, K_{a,b}, wheels, K_{a,b,c},
@@ -51,9 +53,14 @@
  *   orc_superiority      S(d) = llround(2^20 (F_m(d) − λ F_c(d))) (Eq.22; Q20)
  *   orc_objective_eq3    Eq.3 Σ_i |Σ_{v∈B_i} S(v)| with λ folded into S
  *
- * Build: gcc -O2 -std=c11 -ffp-contract=off (Makefile).  Single-threaded.
+ * Build: gcc -O2 -std=c11 -ffp-contract=off -pthread (Makefile).  Single-threaded except
+ * orc_count_forward_mt (sources split over threads, per-thread uint64 partials, SURVEY
+ * §8(c) O4).
  */
+#define _GNU_SOURCE
 #include <math.h>
+#include <pthread.h>
+#include <unistd.h>
 #include <stdint.h>
 #include <stdlib.h>
 #include <string.h>
@@ -81,22 +88,37 @@ static uint64_t edge_key(uint32_t u, uint32_t v) {
 /* O1: simple undirected graph ("undirected graph G=(V,E)")     */
 /* ------------------------------------------------------------------------ */
 
-/* Drops self-loops u==v, maps each sample to its unordered pair (min,max), sorts
- * and removes duplicates (Q1).  edges[] needs room for M keys; returns m, or -1
- * if some id >= n. */
-int64_t orc_simple_graph(const uint32_t *src, const uint32_t *dst, uint64_t M, uint32_t n,
-                         uint64_t *edges) {
+/* Drops self-loops u==v and maps each sample to its unordered pair (min,max) as the key
+ * (min << 32) | max (Q1).  keys[] needs room for M keys; returns the number of keys k, or
+ * -1 if some id >= n.  The keys are then sorted (a library sort, oracle/__init__.py) and
+ * orc_unique_sorted removes the duplicates. */
+int64_t orc_canonical_keys(const uint32_t *src, const uint32_t *dst, uint64_t M, uint32_t n,
+                           uint64_t *keys) {
   uint64_t k = 0;
   for (uint64_t i = 0; i < M; ++i) {
     if (src[i] >= n || dst[i] >= n) return -1;
     if (src[i] == dst[i]) continue;
-    edges[k++] = edge_key(src[i], dst[i]);
+    keys[k++] = edge_key(src[i], dst[i]);
   }
-  qsort(edges, k, sizeof(uint64_t), cmp_u64);
+  return (int64_t)k;
+}
+
+/* Keeps the first of every run of equal keys of an ascending array (in place); returns the
+ * number kept. */
+uint64_t orc_unique_sorted(uint64_t *keys, uint64_t k) {
   uint64_t m = 0;
   for (uint64_t i = 0; i < k; ++i)
-    if (m == 0 || edges[m - 1] != edges[i]) edges[m++] = edges[i];
-  return (int64_t)m;
+    if (m == 0 || keys[m - 1] != keys[i]) keys[m++] = keys[i];
+  return m;
+}
+
+/* O1 in one call (qsort as the sort step; small inputs). */
+int64_t orc_simple_graph(const uint32_t *src, const uint32_t *dst, uint64_t M, uint32_t n,
+                         uint64_t *edges) {
+  int64_t k = orc_canonical_keys(src, dst, M, n, edges);
+  if (k < 0) return -1;
+  qsort(edges, (size_t)k, sizeof(uint64_t), cmp_u64);
+  return (int64_t)orc_unique_sorted(edges, (uint64_t)k);
 }
 
 /* Undirected degree d(v) (Table 1). */
@@ -144,7 +166,7 @@ void orc_direct_degree(const uint64_t *edges, uint64_t m, const uint32_t *deg, u
   }
 }
 
-static void set_edge(const uint64_t *edges, uint8_t *dir, uint8_t *isset, int64_t e, uint32_t from) {
+static void set_edge(const uint64_t *edges, uint8_t *dir, uint8_t *isset, uint64_t e, uint32_t from) {
   uint32_t lo = (uint32_t)(edges[e] >> 32);
   dir[e] = (from == lo) ? 0 : 1;
   isset[e] = 1;
@@ -164,8 +186,9 @@ static void set_edge(const uint64_t *edges, uint8_t *dir, uint8_t *isset, int64_
  * Outputs dir[m]; optional sub[n] (subround in which v was peeled), dsnap[n]
  * (snapshot degree), and counters levels / subrounds.  Returns 0. */
 int orc_direct_paper(const uint64_t *edges, uint64_t m, uint32_t n, const uint64_t *offs,
-                     const uint32_t *adj, uint8_t *dir, uint32_t *sub_out, uint32_t *dsnap_out,
+                     uint8_t *dir, uint32_t *sub_out, uint32_t *dsnap_out,
                      uint32_t *levels_out, uint32_t *subrounds_out) {
+  if (m > UINT32_MAX) return -1; /* edge indices are kept in 32 bits (every config has m < 2^32) */
   size_t nn = n ? n : 1;
   uint32_t *d = (uint32_t *)malloc(sizeof(uint32_t) * nn);        /* residual degree */
   uint32_t *dsnap = (uint32_t *)malloc(sizeof(uint32_t) * nn);
@@ -176,20 +199,16 @@ int orc_direct_paper(const uint64_t *edges, uint64_t m, uint32_t n, const uint64
   uint32_t *frontier = (uint32_t *)malloc(sizeof(uint32_t) * nn);
   uint32_t *next = (uint32_t *)malloc(sizeof(uint32_t) * nn);
   for (uint32_t v = 0; v < n; ++v) d[v] = (uint32_t)(offs[v + 1] - offs[v]);
-  /* N(v) in edge order, each entry with the index of its undirected edge, so that the
-   * "(v,nbr) is unset" test is a direct lookup (the list order does not matter: frontier
-   * members are processed as a set, see readings Q7/Q9). */
-  (void)adj;
+  /* N(v) as the indices of its incident undirected edges, in edge order: the neighbour is
+   * the other end of edges[e], and the "(v,nbr) is unset" test is a direct lookup (the
+   * list order does not matter: frontier members are processed as a set, readings Q7/Q9). */
   uint64_t *cur = (uint64_t *)malloc(sizeof(uint64_t) * nn);
-  uint32_t *nb = (uint32_t *)malloc(sizeof(uint32_t) * (2 * m + 1));
-  uint64_t *eid = (uint64_t *)malloc(sizeof(uint64_t) * (2 * m + 1));
+  uint32_t *eid = (uint32_t *)malloc(sizeof(uint32_t) * (2 * m + 1));
   for (uint32_t v = 0; v < n; ++v) cur[v] = offs[v];
   for (uint64_t i = 0; i < m; ++i) {
     uint32_t u = (uint32_t)(edges[i] >> 32), w = (uint32_t)edges[i];
-    nb[cur[u]] = w;
-    eid[cur[u]++] = i;
-    nb[cur[w]] = u;
-    eid[cur[w]++] = i;
+    eid[cur[u]++] = (uint32_t)i;
+    eid[cur[w]++] = (uint32_t)i;
   }
   free(cur);
 
@@ -213,8 +232,9 @@ int orc_direct_paper(const uint64_t *edges, uint64_t m, uint32_t n, const uint64
       for (uint64_t i = 0; i < nf; ++i) {                 /* line 8 */
         uint32_t v = frontier[i];
         for (uint64_t p = offs[v]; p < offs[v + 1]; ++p) {
-          uint32_t nbr = nb[p];
           uint64_t e = eid[p];
+          uint32_t lo = (uint32_t)(edges[e] >> 32), hi = (uint32_t)edges[e];
+          uint32_t nbr = lo == v ? hi : lo;
           if (isset[e]) continue;
           if (in_frontier[nbr]) {                         /* line 9 */
             int v_first = dsnap[v] < dsnap[nbr] || (dsnap[v] == dsnap[nbr] && v < nbr);
@@ -247,7 +267,7 @@ int orc_direct_paper(const uint64_t *edges, uint64_t m, uint32_t n, const uint64
   if (levels_out) *levels_out = level;
   if (subrounds_out) *subrounds_out = subround;
   free(d); free(dsnap); free(peeled); free(in_frontier); free(queued); free(isset);
-  free(frontier); free(next); free(nb); free(eid);
+  free(frontier); free(next); free(eid);
   return 0;
 }
 
@@ -485,25 +505,28 @@ void orc_cost_eq1(uint32_t n, uint64_t m, const uint32_t *od, uint64_t *lo, uint
 /* Oriented, relabelled CSR (directed graph G; relabel P:450 line 16-20) */
 /* ------------------------------------------------------------------------ */
 
-void orc_oriented_csr(const uint64_t *edges, uint64_t m, uint32_t n, const uint8_t *dir,
-                      const uint32_t *perm, uint64_t *offs, uint32_t *col) {
-  uint64_t *fill = (uint64_t *)calloc(n ? n : 1, sizeof(uint64_t));
-  for (uint64_t i = 0; i < m; ++i) {
-    uint32_t u = (uint32_t)(edges[i] >> 32), v = (uint32_t)edges[i];
-    uint32_t s = dir[i] ? v : u;
-    fill[perm[s]]++;
-  }
-  offs[0] = 0;
-  for (uint32_t x = 0; x < n; ++x) offs[x + 1] = offs[x] + fill[x];
-  for (uint32_t x = 0; x < n; ++x) fill[x] = offs[x];
+/* Directed edge i as the key (perm[source] << 32) | perm[target]: sorting these keys
+ * (a library sort, oracle/__init__.py) groups every out-list N+(x) by its new label x, each
+ * list ascending. */
+void orc_oriented_keys(const uint64_t *edges, uint64_t m, const uint8_t *dir, const uint32_t *perm,
+                       uint64_t *keys) {
   for (uint64_t i = 0; i < m; ++i) {
     uint32_t u = (uint32_t)(edges[i] >> 32), v = (uint32_t)edges[i];
     uint32_t s = dir[i] ? v : u, t = dir[i] ? u : v;
-    col[fill[perm[s]]++] = perm[t];
+    keys[i] = ((uint64_t)perm[s] << 32) | perm[t];
   }
-  for (uint32_t x = 0; x < n; ++x)
-    qsort(col + offs[x], offs[x + 1] - offs[x], sizeof(uint32_t), cmp_u32);
-  free(fill);
+}
+
+/* CSR of ascending (source << 32) | target keys: offs[x] = number of keys with source < x,
+ * col[i] = target of key i. */
+void orc_csr_from_sorted_keys(const uint64_t *keys, uint64_t m, uint32_t n, uint64_t *offs,
+                              uint32_t *col) {
+  memset(offs, 0, sizeof(uint64_t) * ((size_t)n + 1));
+  for (uint64_t i = 0; i < m; ++i) {
+    offs[(keys[i] >> 32) + 1]++;
+    col[i] = (uint32_t)keys[i];
+  }
+  for (uint32_t x = 0; x < n; ++x) offs[x + 1] += offs[x];
 }
 
 /* ------------------------------------------------------------------------ */
@@ -624,28 +647,100 @@ int orc_local_triangles(const uint32_t *src, const uint32_t *dst, uint64_t M, co
 /* is counted once at its unique source u with u->v, u->w, v->w.       */
 /* ------------------------------------------------------------------------ */
 
-/* Counts over u in [u_begin, u_end).  tv (per label of the CSR, may be NULL)
- * gets +1 at all three corners of every triangle found. */
+/* The triangles counted at one source u: for every v in N+(u), |N+(u) ∩ N+(v)| by a
+ * two-pointer merge of the two ascending lists.  tv (per label of the CSR, may be NULL)
+ * gets +1 at all three corners of every triangle found (atomically: sources run on
+ * several threads). */
+static uint64_t count_source(uint32_t u, const uint64_t *offs, const uint32_t *col, uint64_t *tv) {
+  uint64_t T = 0;
+  for (uint64_t p = offs[u]; p < offs[u + 1]; ++p) {
+    uint32_t v = col[p];
+    uint64_t i = offs[u], ie = offs[u + 1], j = offs[v], je = offs[v + 1];
+    while (i < ie && j < je) {
+      if (col[i] < col[j]) ++i;
+      else if (col[i] > col[j]) ++j;
+      else {
+        ++T;
+        if (tv) {
+          __atomic_fetch_add(&tv[u], 1, __ATOMIC_RELAXED);
+          __atomic_fetch_add(&tv[v], 1, __ATOMIC_RELAXED);
+          __atomic_fetch_add(&tv[col[i]], 1, __ATOMIC_RELAXED);
+        }
+        ++i; ++j;
+      }
+    }
+  }
+  return T;
+}
+
+/* Sources u in [u_begin, u_end) are handed out in chunks of COUNT_CHUNK from a shared
+ * counter; every thread sums its own uint64 partial and the partials are added at the
+ * end (integer addition: the result does not depend on the split). */
+#define COUNT_CHUNK 256
+typedef struct {
+  const uint64_t *offs;
+  const uint32_t *col;
+  uint64_t *tv;
+  uint32_t u_begin, u_end;
+  uint64_t next_chunk; /* shared, atomic */
+} count_job;
+
+typedef struct {
+  count_job *job;
+  uint64_t T;
+} count_worker_arg;
+
+static void *count_worker(void *p) {
+  count_worker_arg *a = (count_worker_arg *)p;
+  count_job *J = a->job;
+  uint64_t T = 0;
+  for (;;) {
+    uint64_t c = __atomic_fetch_add(&J->next_chunk, 1, __ATOMIC_RELAXED);
+    uint64_t lo = (uint64_t)J->u_begin + c * COUNT_CHUNK;
+    if (lo >= J->u_end) break;
+    uint64_t hi = lo + COUNT_CHUNK < J->u_end ? lo + COUNT_CHUNK : J->u_end;
+    for (uint64_t u = lo; u < hi; ++u) T += count_source((uint32_t)u, J->offs, J->col, J->tv);
+  }
+  a->T = T;
+  return NULL;
+}
+
+/* T over sources [u_begin, u_end) on `threads` threads (<= 0: all online cores). */
+uint64_t orc_count_forward_mt(uint32_t n, const uint64_t *offs, const uint32_t *col, uint32_t u_begin,
+                              uint32_t u_end, uint64_t *tv, int threads) {
+  if (u_end > n) u_end = n;
+  if (u_begin >= u_end) return 0;
+  if (threads <= 0) threads = (int)sysconf(_SC_NPROCESSORS_ONLN);
+  if (threads < 1) threads = 1;
+  count_job J = {offs, col, tv, u_begin, u_end, 0};
+  pthread_t *th = (pthread_t *)malloc(sizeof(pthread_t) * threads);
+  count_worker_arg *args = (count_worker_arg *)malloc(sizeof(count_worker_arg) * threads);
+  int started = 0;
+  for (int t = 0; t < threads; ++t) {
+    args[t].job = &J;
+    args[t].T = 0;
+    if (t > 0 && pthread_create(&th[t], NULL, count_worker, &args[t]) == 0) ++started;
+    else if (t > 0) args[t].job = NULL; /* not started: its share is taken by the others */
+  }
+  count_worker(&args[0]);
+  uint64_t T = args[0].T;
+  for (int t = 1; t < threads; ++t) {
+    if (!args[t].job) continue;
+    pthread_join(th[t], NULL);
+    T += args[t].T;
+  }
+  (void)started;
+  free(th);
+  free(args);
+  return T;
+}
+
+/* Single-threaded entry point (small graphs, range checks). */
 uint64_t orc_count_forward(uint32_t n, const uint64_t *offs, const uint32_t *col, uint32_t u_begin,
                            uint32_t u_end, uint64_t *tv) {
   uint64_t T = 0;
   if (u_end > n) u_end = n;
-  for (uint32_t u = u_begin; u < u_end; ++u) {
-    for (uint64_t p = offs[u]; p < offs[u + 1]; ++p) {
-      uint32_t v = col[p];
-      /* |N+(u) ∩ N+(v)| by two-pointer merge of two ascending lists */
-      uint64_t i = offs[u], ie = offs[u + 1], j = offs[v], je = offs[v + 1];
-      while (i < ie && j < je) {
-        if (col[i] < col[j]) ++i;
-        else if (col[i] > col[j]) ++j;
-        else {
-          ++T;
-          if (tv) { tv[u]++; tv[v]++; tv[col[i]]++; }
-          ++i; ++j;
-        }
-      }
-    }
-  }
+  for (uint32_t u = u_begin; u < u_end; ++u) T += count_source(u, offs, col, tv);
   return T;
 }
 

@@ -9,7 +9,7 @@ CPU fallback: if ``libtc_b200.so`` is missing or no CUDA device is present the
 calls raise.
 
 Low-level names mirror the C-ABI (``tc_graph_from_edges``, ``tc_direct``,
-``tc_reorder``, ``tc_count``, ``tc_count_range``, ``tc_partition``,
+``tc_reorder``, ``tc_reorder_dist``, ``tc_count``, ``tc_count_range``, ``tc_partition``,
 ``tc_count_dist``, ...); :class:`Graph` is a small convenience wrapper.
 """
 from __future__ import annotations
@@ -51,7 +51,7 @@ class Stats(ctypes.Structure):
         ("ms_build", ctypes.c_double), ("ms_direct", ctypes.c_double),
         ("ms_reorder", ctypes.c_double), ("ms_count", ctypes.c_double),
         ("ms_count_kernel", ctypes.c_double), ("count_launches", ctypes.c_uint64),
-        ("eq3_units", ctypes.c_int64), ("nunits", ctypes.c_uint64)]
+        ("eq3_units", ctypes.c_int64), ("nunits", ctypes.c_uint64), ("unit_buckets", ctypes.c_uint64)]
 
     def as_dict(self):
         d = {f: getattr(self, f) for f, _ in self._fields_}
@@ -76,6 +76,7 @@ def lib():
             "tc_graph_from_edges": [p, p, u64, u32, i32, p, pp],
             "tc_direct": [p, i32],
             "tc_reorder": [p, i32, p],
+            "tc_reorder_dist": [p, i32, p, p, i32, i32],
             "tc_set_schedule": [p, i32],
             "tc_count": [p, p, p],
             "tc_count_range": [p, u32, u32, p, p],
@@ -174,6 +175,12 @@ def make_aorder_params(k=32, lam=9.682, alpha=0.5, beta=0.5, bw=None, order=0):
 def tc_reorder(g, rule, params=None):
     _check(lib().tc_reorder(g, REORDER[rule] if isinstance(rule, str) else rule,
                             None if params is None else ctypes.byref(params)))
+
+
+def tc_reorder_dist(g, rule, params, comm, rank, world):
+    """tc_reorder on replicas: the A-order greedy on rank 0, pi broadcast over NCCL."""
+    _check(lib().tc_reorder_dist(g, REORDER[rule] if isinstance(rule, str) else rule,
+                                 None if params is None else ctypes.byref(params), comm, rank, world))
 
 
 def tc_set_schedule(g, sched):
@@ -380,16 +387,15 @@ class Graph:
         tc_export_buckets(self._h, b)
         return b
 
-    def export_units(self, k=32):
-        """Edge-unit A-order (schedule "edge_aorder"): (units in bucket order, offsets)."""
-        # sized generously: units <= sum_u ceil(d~(u)/32) <= m, buckets = ceil(units / k)
+    def export_units(self):
+        """Edge-unit A-order (schedule "edge_aorder"): (units in bucket order as
+        (u << 32) | j, bucket offsets); sizes from the library's own statistics."""
         m = self.stats()["m"]
         u = np.zeros(max(m, 1), dtype=np.uint64)
         off = np.zeros(max(m, 1) + 2, dtype=np.uint32)
         tc_export_units(self._h, u, off)
-        nu = self.stats()["nunits"]
-        nb = (nu + k - 1) // k
-        return u[:nu], off[:nb + 1]
+        st = self.stats()
+        return u[:st["nunits"]], off[:st["unit_buckets"] + 1]
 
 
 def count_triangles(src, dst, num_vertices, direct="degree", reorder="none", per_vertex=False,

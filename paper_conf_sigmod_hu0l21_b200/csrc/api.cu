@@ -130,13 +130,14 @@ namespace nccl {
 typedef int Result;
 typedef struct Comm *Comm_t;
 struct UniqueId { char internal[128]; };
-enum { Uint64 = 5 };
+enum { Uint32 = 3, Uint64 = 5 };
 enum { Sum = 0 };
 struct Api {
   void *h = nullptr;
   Result (*GetUniqueId)(UniqueId *) = nullptr;
   Result (*CommInitRank)(Comm_t *, int, UniqueId, int) = nullptr;
   Result (*AllReduce)(const void *, void *, size_t, int, int, Comm_t, cudaStream_t) = nullptr;
+  Result (*Broadcast)(const void *, void *, size_t, int, int, Comm_t, cudaStream_t) = nullptr;
   Result (*CommDestroy)(Comm_t) = nullptr;
   const char *(*GetErrorString)(Result) = nullptr;
 };
@@ -150,10 +151,11 @@ static Api &api() {
     a.GetUniqueId = (Result(*)(UniqueId *))dlsym(a.h, "ncclGetUniqueId");
     a.CommInitRank = (Result(*)(Comm_t *, int, UniqueId, int))dlsym(a.h, "ncclCommInitRank");
     a.AllReduce = (Result(*)(const void *, void *, size_t, int, int, Comm_t, cudaStream_t))dlsym(a.h, "ncclAllReduce");
+    a.Broadcast = (Result(*)(const void *, void *, size_t, int, int, Comm_t, cudaStream_t))dlsym(a.h, "ncclBroadcast");
     a.CommDestroy = (Result(*)(Comm_t))dlsym(a.h, "ncclCommDestroy");
     a.GetErrorString = (const char *(*)(Result))dlsym(a.h, "ncclGetErrorString");
   });
-  TC_REQUIRE(a.h && a.GetUniqueId && a.CommInitRank && a.AllReduce && a.CommDestroy, ST_NCCL,
+  TC_REQUIRE(a.h && a.GetUniqueId && a.CommInitRank && a.AllReduce && a.Broadcast && a.CommDestroy, ST_NCCL,
              "libnccl.so.2 not loadable");
   return a;
 }
@@ -285,6 +287,76 @@ tc_status tc_reorder(tc_graph *gp, tc_reorder_rule rule, const tc_aorder_params 
   });
 }
 
+namespace {
+// A-order computed once (rank `root`) and broadcast: a 2-word header [b + 1, eq3], then pi
+// (n u32) and bucket_off (b + 1 u32), all on the graph's stream (a11 plumbing).
+struct BroadcastAOrder : AOrderSource {
+  nccl::Comm_t comm;
+  int rank, root = 0;
+  bool produce(Graph &g, const std::vector<uint32_t> &h_od, const tc_aorder_params &p) override {
+    nccl::Api &a = nccl::api();
+    cudaStream_t s = g.stream;
+    const uint32_t n = g.n;
+    std::vector<uint32_t> h_perm;
+    uint64_t hdr[2] = {0, 0};
+    if (rank == root) {
+      aorder_host(h_od, p, h_perm, g.h_bucket_off, g.eq3);
+      hdr[0] = g.h_bucket_off.size();
+      hdr[1] = (uint64_t)g.eq3;
+    }
+    DevBuf<uint64_t> dh;
+    dh.alloc(2, s);
+    TC_CUDA(cudaMemcpyAsync(dh.get(), hdr, sizeof(hdr), cudaMemcpyHostToDevice, s));
+    nccl::check(a.Broadcast(dh.get(), dh.get(), 2, nccl::Uint64, root, comm, s), "ncclBroadcast(header)");
+    TC_CUDA(cudaMemcpyAsync(hdr, dh.get(), sizeof(hdr), cudaMemcpyDeviceToHost, s));
+    TC_CUDA(cudaStreamSynchronize(s));
+    const size_t nb1 = (size_t)hdr[0];
+    TC_REQUIRE(nb1 >= 1, ST_NCCL, "A-order broadcast: empty bucket table");
+    if (rank != root) {
+      g.h_bucket_off.assign(nb1, 0);
+      g.eq3 = (int64_t)hdr[1];
+    }
+    if (n) g.perm.alloc(n, s);
+    g.bucket_off.alloc(nb1, s);
+    if (rank == root) {
+      if (n) TC_CUDA(cudaMemcpyAsync(g.perm.get(), h_perm.data(), sizeof(uint32_t) * n, cudaMemcpyHostToDevice, s));
+      TC_CUDA(cudaMemcpyAsync(g.bucket_off.get(), g.h_bucket_off.data(), sizeof(uint32_t) * nb1,
+                              cudaMemcpyHostToDevice, s));
+    }
+    if (n) nccl::check(a.Broadcast(g.perm.get(), g.perm.get(), n, nccl::Uint32, root, comm, s), "ncclBroadcast(pi)");
+    nccl::check(a.Broadcast(g.bucket_off.get(), g.bucket_off.get(), nb1, nccl::Uint32, root, comm, s),
+                "ncclBroadcast(bucket_off)");
+    if (rank != root)
+      TC_CUDA(cudaMemcpyAsync(g.h_bucket_off.data(), g.bucket_off.get(), sizeof(uint32_t) * nb1,
+                              cudaMemcpyDeviceToHost, s));
+    TC_CUDA(cudaStreamSynchronize(s));  // host vectors must outlive the copies
+    return true;
+  }
+};
+}  // namespace
+
+tc_status tc_reorder_dist(tc_graph *gp, tc_reorder_rule rule, const tc_aorder_params *p, void *comm, int rank,
+                          int world) {
+  return guard([&] {
+    Graph &g = checked(gp, G_DIRECTED);
+    TC_REQUIRE(rule >= TC_REORDER_NONE && rule <= TC_REORDER_PAPER, ST_INVALID, "unknown reorder rule");
+    TC_REQUIRE(comm != nullptr, ST_INVALID, "comm is NULL");
+    TC_REQUIRE(world >= 1 && rank >= 0 && rank < world, ST_INVALID, "bad rank/world");
+    tc_aorder_params prm = defaults_or(p);
+    g.abw.assign(prm.bw ? prm.bw : nullptr, prm.bw ? prm.bw + prm.bw_len : nullptr);
+    g.aparams = prm;
+    g.aparams.bw = g.abw.empty() ? nullptr : g.abw.data();
+    g.aparams_set = true;
+    StageTimer t(g.stream);
+    BroadcastAOrder src;
+    src.comm = (nccl::Comm_t)comm;
+    src.rank = rank;
+    reorder_graph(g, rule, prm, rule == TC_REORDER_PAPER ? &src : nullptr);
+    g.ms_reorder = t.stop();
+    gp->partitions.clear();
+  });
+}
+
 tc_status tc_set_schedule(tc_graph *gp, tc_schedule s) {
   return guard([&] {
     TC_REQUIRE(gp != nullptr, ST_INVALID, "graph is NULL");
@@ -319,12 +391,16 @@ static uint64_t do_count(tc_graph *gp, uint32_t ub, uint32_t ue, uint64_t *per_v
   }
   float kms = 0;
   uint64_t launches = 0;
-  uint64_t T = count_graph(g, ub, ue, per_vertex ? tnew.get() : nullptr, g_opt_profile ? &kms : nullptr, &launches);
+  uint64_t T = 0;
+  DevBuf<unsigned long long> dT;  // a11: the allreduce consumes the device partial directly
+  if (reduce) {
+    dT.alloc(1, g.stream);
+    TC_CUDA(cudaMemsetAsync(dT.get(), 0, 8, g.stream));
+  }
+  T = count_graph(g, ub, ue, per_vertex ? tnew.get() : nullptr, g_opt_profile ? &kms : nullptr, &launches, -1,
+                  reduce ? dT.get() : nullptr);
   if (reduce) {
     nccl::Api &a = nccl::api();
-    DevBuf<uint64_t> dT;
-    dT.alloc(1, g.stream);
-    TC_CUDA(cudaMemcpyAsync(dT.get(), &T, 8, cudaMemcpyHostToDevice, g.stream));
     nccl::check(a.AllReduce(dT.get(), dT.get(), 1, nccl::Uint64, nccl::Sum, (nccl::Comm_t)comm, g.stream),
                 "ncclAllReduce(T)");
     if (per_vertex && g.n)
@@ -507,6 +583,7 @@ tc_status tc_get_stats(const tc_graph *gp, tc_stats_t *o) {
     o->count_launches = g.count_launches;
     o->eq3_units = g.units_ready ? g.eq3_units : -1;
     o->nunits = g.units_ready && !g.h_unit_off.empty() ? g.h_unit_off.back() : 0;
+    o->unit_buckets = g.units_ready && !g.h_unit_off.empty() ? g.h_unit_off.size() - 1 : 0;
   });
 }
 

@@ -792,63 +792,38 @@ __global__ __launch_bounds__(BM_THREADS) void count_bitmap_kernel(const uint64_t
   block_add_u64(acc, T);
 }
 
-// ---- edge-unit A-order (TC_SCHED_EDGE_AORDER)
-// Units = the (u, 32-v chunk) work items, u ascending, chunks ascending (d~(u) >= 2).
-// nitems[u] = ceil(d~(u) / 32) for d~(u) >= 2.
-__global__ void unit_count_kernel(const uint64_t *__restrict__ offs, uint32_t n, uint32_t *__restrict__ cnt) {
-  for (uint64_t u = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; u < n; u += (uint64_t)gridDim.x * blockDim.x) {
-    const uint32_t d = (uint32_t)(offs[u + 1] - offs[u]);
-    cnt[u] = d >= 2 ? (d + SV - 1) / SV : 0u;
-  }
-}
-// Warp per source: item (u, c0) gets S = sum over its edges u->v of S(d~(v)) (table in
-// fixed point, 0 for d~(v) = 0) and active = some d~(v) >= 1 (it has wedges).
+// ---- edge-unit A-order (TC_SCHED_EDGE_AORDER, Q26)
+// A unit is ONE directed edge u -> v (CSR position p, index j = p - offs[u]); its task
+// streams N+(v) and binary-searches every w in N+(u).  Superiority S(d~(v)) (the streamed
+// list); d~(v) = 0 -> no work, inactive.  Warp per source: lanes over its out-edges.
 __global__ void unit_sup_kernel(const uint64_t *__restrict__ offs, const uint32_t *__restrict__ col, uint32_t n,
-                                const uint64_t *__restrict__ ioff, const int64_t *__restrict__ stab,
-                                uint64_t *__restrict__ items, int64_t *__restrict__ isup,
-                                uint8_t *__restrict__ iact) {
+                                const int64_t *__restrict__ stab, uint64_t *__restrict__ items,
+                                int64_t *__restrict__ isup, uint8_t *__restrict__ iact) {
   const uint64_t nw = (uint64_t)gridDim.x * (blockDim.x / 32);
   for (uint64_t u = (uint64_t)blockIdx.x * (blockDim.x / 32) + warp_id(); u < n; u += nw) {
     const uint64_t a = offs[u];
     const uint32_t d = (uint32_t)(offs[u + 1] - a);
-    if (d < 2) continue;
-    const uint64_t base = ioff[u];
-    for (uint32_t c = 0; c * SV < d; ++c) {
-      const uint32_t j = c * SV + lane_id();
-      int64_t sv = 0;
-      bool act = false;
-      if (j < d) {
-        const uint32_t v = col[a + j];
-        const uint32_t dv = (uint32_t)(offs[v + 1] - offs[v]);
-        if (dv) {
-          sv = stab[dv];
-          act = true;
-        }
-      }
-#pragma unroll
-      for (int o = 16; o > 0; o >>= 1) sv += __shfl_xor_sync(0xffffffffu, sv, o);
-      const unsigned any = __ballot_sync(0xffffffffu, act);
-      if (lane_id() == 0) {
-        items[base + c] = (u << 32) | (uint64_t)(c * SV);
-        isup[base + c] = sv;
-        iact[base + c] = any ? 1 : 0;
-      }
+    for (uint32_t j = lane_id(); j < d; j += 32) {
+      const uint32_t v = col[a + j];
+      const uint32_t dv = (uint32_t)(offs[v + 1] - offs[v]);
+      items[a + j] = (u << 32) | (uint64_t)j;
+      isup[a + j] = dv ? stab[dv] : 0;
+      iact[a + j] = dv ? 1 : 0;
     }
   }
 }
-// CTA per bucket of units (fetched dynamically); the bucket's items dealt to the warps.
+// CTA per bucket of edge units (fetched dynamically); warp per unit: the lanes stream
+// N+(v) and binary-search each w in N+(u) in global memory (Fox's edge-centric pattern,
+// no staging: a bucket's edges have unrelated sources).  MODE 1: +1 at u, v, w per
+// triangle; MODE 2: +1 at the CSR positions of (u,v), (u,w), (v,w).
 template <int MODE>
 __global__ __launch_bounds__(CT_THREADS) void count_units_kernel(const uint64_t *__restrict__ offs,
                                                                  const uint32_t *__restrict__ col,
                                                                  const uint64_t *__restrict__ units,
                                                                  const uint32_t *__restrict__ uoff, uint32_t nb,
-                                                                 uint32_t ub, uint32_t ue, uint32_t cap,
-                                                                 unsigned *bucket_ctr, unsigned long long *T,
-                                                                 unsigned long long *tv) {
-  __shared__ WarpScratch s_ws[CT_WARPS];
+                                                                 uint32_t ub, uint32_t ue, unsigned *bucket_ctr,
+                                                                 unsigned long long *T, unsigned long long *tv) {
   __shared__ uint32_t s_bucket;
-  const uint32_t slice = warp_id() * warp_stride(cap, MODE == 1 || MODE == 2);
-  WarpScratch &ws = s_ws[warp_id()];
   uint64_t acc = 0;
   while (true) {
     __syncthreads();
@@ -858,9 +833,36 @@ __global__ __launch_bounds__(CT_THREADS) void count_units_kernel(const uint64_t 
     if (bi >= nb) break;
     for (uint32_t i = uoff[bi] + warp_id(); i < uoff[bi + 1]; i += CT_WARPS) {
       const uint64_t it = units[i];
-      const uint32_t u = (uint32_t)(it >> 32);
+      const uint32_t u = (uint32_t)(it >> 32), j = (uint32_t)it;
       if (u < ub || u >= ue) continue;  // tc_count_range / tc_count_dist slices
-      acc += warp_item<MODE>(offs, col, u, (uint32_t)it, slice, cap, ws, tv);
+      const uint64_t a = offs[u];
+      const uint32_t L = (uint32_t)(offs[u + 1] - a);
+      if (L < 2) continue;
+      const uint32_t v = col[a + j];
+      const uint64_t vb = offs[v];
+      const uint32_t dv = (uint32_t)(offs[v + 1] - vb);
+      const GlobalSearch search{col + a, L, 0};
+      uint32_t cnt = 0;
+      for (uint32_t t = lane_id(); t < dv; t += 32) {
+        const uint32_t w = col[vb + t];
+        uint32_t pos;
+        const bool hit = search(w, pos);
+        cnt += hit ? 1u : 0u;
+        if (MODE == 1 && hit) {
+          atomicAdd(&tv[v], 1ull);
+          atomicAdd(&tv[w], 1ull);
+        }
+        if (MODE == 2 && hit) {
+          atomicAdd(&tv[a + j], 1ull);
+          atomicAdd(&tv[a + pos], 1ull);
+          atomicAdd(&tv[vb + t], 1ull);
+        }
+      }
+      if (MODE == 1) {
+        const uint32_t tot = warp_sum((uint64_t)cnt);
+        if (lane_id() == 0 && tot) atomicAdd(&tv[u], (unsigned long long)tot);
+      }
+      acc += cnt;
     }
   }
   block_add_u64(acc, T);
@@ -949,9 +951,24 @@ __global__ void bounds_kernel(const uint64_t *__restrict__ pre, uint32_t n, uint
 
 }  // namespace
 
-static void configure_kernels() {
-  static bool done = false;
-  if (done) return;
+// Per-device setup: the >48 KB dynamic shared-memory opt-in (cudaFuncSetAttribute) and the
+// __constant__ options are per device, so both are tracked per device under a mutex.
+static std::mutex g_cfg_mu;
+struct DeviceCfg {
+  bool configured = false;
+  int bracket = 1, intersect = 0, extra = -1;
+};
+static DeviceCfg g_cfg[64];
+
+static DeviceCfg &device_cfg() {
+  int dev = 0;
+  TC_CUDA(cudaGetDevice(&dev));
+  TC_REQUIRE(dev >= 0 && dev < 64, ST_CUDA, "device ordinal >= 64");
+  return g_cfg[dev];
+}
+
+static void configure_kernels_locked(DeviceCfg &c) {
+  if (c.configured) return;
   size_t large_smem = LG_SMEM_WORDS * sizeof(uint32_t);
   for (auto fn : {count_large_kernel<0>, count_large_kernel<1>, count_large_kernel<2>})
     TC_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)large_smem));
@@ -961,11 +978,28 @@ static void configure_kernels() {
     TC_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, small_max));
   for (auto fn : {count_range_kernel<0>, count_range_kernel<1>, count_range_kernel<2>})
     TC_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, small_max));
-  for (auto fn : {count_units_kernel<0>, count_units_kernel<1>, count_units_kernel<2>})
-    TC_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, small_max));
   TC_CUDA(cudaFuncSetAttribute(count_bitmap_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                (int)(BM_SMEM_MAX_N / 8)));
-  done = true;
+  c.configured = true;
+}
+
+// kernel attributes + the option constants of the current device, once per change
+static void configure_kernels() {
+  std::lock_guard<std::mutex> lk(g_cfg_mu);
+  DeviceCfg &c = device_cfg();
+  configure_kernels_locked(c);
+  if (g_opt_extra != c.extra && g_opt_extra >= 0) {
+    TC_CUDA(cudaMemcpyToSymbol(g_extra, &g_opt_extra, sizeof(int)));
+    c.extra = g_opt_extra;
+  }
+  if (g_opt_bracket != c.bracket) {
+    TC_CUDA(cudaMemcpyToSymbol(g_bracket, &g_opt_bracket, sizeof(int)));
+    c.bracket = g_opt_bracket;
+  }
+  if (g_opt_intersect != c.intersect) {
+    TC_CUDA(cudaMemcpyToSymbol(g_merge, &g_opt_intersect, sizeof(int)));
+    c.intersect = g_opt_intersect;
+  }
 }
 
 // L2 access-policy window over the head of the CSR allocation [offs | col...] for the
@@ -1037,33 +1071,24 @@ static int occupancy(const void *fn, int threads, size_t smem) {
 }
 
 uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *kernel_ms, uint64_t *launches,
-                     int mode) {
+                     int mode, unsigned long long *d_T) {
   // 0 count, 1 per-vertex (t[n], new labels), 2 per-edge (CSR positions), 3 count with
   // g_opt_extra extra searches per wedge in the warp-item kernel (§5.3 experiment)
   if (mode < 0) mode = d_tv ? 1 : (g_opt_extra >= 0 ? 3 : 0);
   const bool pv = mode == 1 || mode == 2;
   cudaStream_t s = g.stream;
   configure_kernels();
-  {
-    static int last_bracket = 1, last_intersect = 0, last_extra = -1;
-    if (g_opt_extra != last_extra && g_opt_extra >= 0) {
-      TC_CUDA(cudaMemcpyToSymbol(g_extra, &g_opt_extra, sizeof(int)));
-      last_extra = g_opt_extra;
-    }
-    if (g_opt_bracket != last_bracket) {
-      TC_CUDA(cudaMemcpyToSymbol(g_bracket, &g_opt_bracket, sizeof(int)));
-      last_bracket = g_opt_bracket;
-    }
-    if (g_opt_intersect != last_intersect) {
-      TC_CUDA(cudaMemcpyToSymbol(g_merge, &g_opt_intersect, sizeof(int)));
-      last_intersect = g_opt_intersect;
-    }
-  }
   if (ue > g.n) ue = g.n;
   uint64_t nlaunch = 0;
-  DevBuf<unsigned long long> dT;
-  dT.alloc(1, s);
-  TC_CUDA(cudaMemsetAsync(dT.get(), 0, sizeof(unsigned long long), s));
+  DevBuf<unsigned long long> dT_own;
+  if (!d_T) {
+    dT_own.alloc(1, s);
+    TC_CUDA(cudaMemsetAsync(dT_own.get(), 0, sizeof(unsigned long long), s));
+  }
+  struct {
+    unsigned long long *p;
+    unsigned long long *get() const { return p; }
+  } dT{d_T ? d_T : dT_own.get()};
   unsigned long long *tv = reinterpret_cast<unsigned long long *>(d_tv);
   const uint32_t cap = (uint32_t)g_opt_small_cap;
   int sched = g.schedule;
@@ -1106,8 +1131,7 @@ uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *
     build_units(g);
     const uint32_t nb = (uint32_t)g.h_unit_off.size() - 1;
     if (nb) {
-      const uint32_t rcap = fit_cap(cap, pv);
-      size_t smem = (size_t)CT_WARPS * warp_stride(rcap, pv) * sizeof(uint32_t);
+      const size_t smem = 0;
       auto fn = mode == 2 ? count_units_kernel<2> : mode == 1 ? count_units_kernel<1> : count_units_kernel<0>;
       int occ = occupancy((const void *)fn, CT_THREADS, smem);
       unsigned grid = (unsigned)std::min<uint64_t>(nb, (uint64_t)num_sms() * occ);
@@ -1116,7 +1140,7 @@ uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *
       TC_CUDA(cudaMemsetAsync(bctr.get(), 0, sizeof(unsigned), s));
       if (kernel_ms) TC_CUDA(cudaEventRecord(e0, s));
       ProfScope prof("count_units", s, 0.0);
-      fn<<<grid, CT_THREADS, smem, s>>>(g.offs.get(), g.col.get(), g.units.get(), g.unit_off.get(), nb, ub, ue, rcap,
+      fn<<<grid, CT_THREADS, smem, s>>>(g.offs.get(), g.col.get(), g.units.get(), g.unit_off.get(), nb, ub, ue,
                                         bctr.get(), dT.get(), tv);
       TC_LAUNCH_CHECK();
       if (kernel_ms) TC_CUDA(cudaEventRecord(e1, s));
@@ -1168,9 +1192,9 @@ uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *
       TC_LAUNCH_CHECK();
       // the item list is scattered before the host reads the bin sizes back (the scatter
       // needs only the device-side cursors), into a buffer sized by the bound
-      // sum_u ceil(d~(u)/32) <= m/32 + #sources
+      // sum_u ceil(d~(u)/32) <= m/32 + #{sources with d~ >= 2} <= m/32 + min(#sources, m/2)
       DevBuf<uint64_t> items;
-      items.alloc(g.m / SV + (uint64_t)(ue - ub) + 1, s);
+      items.alloc(g.m / SV + std::min<uint64_t>((uint64_t)(ue - ub), g.m / 2) + 1, s);
       {
         uint64_t span = 256ull * SC_PER_THREAD;
         unsigned grid = (unsigned)std::min<uint64_t>((ue - ub + span - 1) / span, (uint64_t)num_sms() * 8);
@@ -1239,7 +1263,7 @@ uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *
     }
   }
   uint64_t hT = 0;
-  TC_CUDA(cudaMemcpyAsync(&hT, dT.get(), sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
+  if (!d_T) TC_CUDA(cudaMemcpyAsync(&hT, dT.get(), sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
   TC_CUDA(cudaStreamSynchronize(s));
   if (kernel_ms) {
     float ms = 0;
@@ -1252,9 +1276,9 @@ uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *
   return hT;
 }
 
-// Edge-unit A-order: units and their superiority on the GPU, Algorithm 2 over the units on
-// the host (aorder_units, the same greedy as the vertex A-order), units uploaded in bucket
-// order.  Inactive units (no wedge) are dropped: they add nothing to T.
+// Edge-unit A-order: one unit per directed edge, superiority on the GPU, Algorithm 2 over the
+// units on the host (aorder_units, the same greedy as the vertex A-order), active units
+// uploaded in bucket order.  Inactive units (d~(v) = 0) are dropped: they add nothing to T.
 void build_units(Graph &g) {
   if (g.units_ready) return;
   cudaStream_t s = g.stream;
@@ -1268,18 +1292,7 @@ void build_units(Graph &g) {
     prm.k = 32;
     prm.order = 0;
   }
-  DevBuf<uint32_t> cnt;
-  DevBuf<uint64_t> ioff;
-  cnt.alloc(n ? n : 1, s);
-  ioff.alloc((uint64_t)n + 1, s);
-  if (n) {
-    unit_count_kernel<<<grid_for(n, 256), 256, 0, s>>>(g.offs.get(), n, cnt.get());
-    TC_LAUNCH_CHECK();
-  }
-  scan_u32_to_u64(cnt.get(), ioff.get(), n, s);
-  uint64_t nitems = 0;
-  TC_CUDA(cudaMemcpyAsync(&nitems, ioff.get() + n, 8, cudaMemcpyDeviceToHost, s));
-  TC_CUDA(cudaStreamSynchronize(s));
+  const uint64_t nitems = g.m;
   // superiority per out-degree value (fixed point, λ folded in); max d~ is label-free
   ensure_od(g);
   const uint32_t maxd = g.max_outdeg;
@@ -1294,7 +1307,7 @@ void build_units(Graph &g) {
   isup.alloc(nitems ? nitems : 1, s);
   iact.alloc(nitems ? nitems : 1, s);
   if (nitems) {
-    unit_sup_kernel<<<grid_for((uint64_t)n * 32, 256), 256, 0, s>>>(g.offs.get(), g.col.get(), n, ioff.get(), stab.get(),
+    unit_sup_kernel<<<grid_for((uint64_t)n * 32, 256), 256, 0, s>>>(g.offs.get(), g.col.get(), n, stab.get(),
                                                                     items.get(), isup.get(), iact.get());
     TC_LAUNCH_CHECK();
   }
@@ -1356,7 +1369,7 @@ void partition_graph(Graph &g, uint32_t world, uint32_t *bounds) {
     TC_LAUNCH_CHECK();
   }
   scan_u64(w.get(), pre.get(), n, s);
-  bounds_kernel<<<1, 1024, 0, s>>>(pre.get(), n, world, db.get());
+  bounds_kernel<<<grid_for((uint64_t)world + 1, 256), 256, 0, s>>>(pre.get(), n, world, db.get());
   TC_LAUNCH_CHECK();
   TC_CUDA(cudaMemcpyAsync(bounds, db.get(), sizeof(uint32_t) * (world + 1), cudaMemcpyDeviceToHost, s));
   TC_CUDA(cudaStreamSynchronize(s));

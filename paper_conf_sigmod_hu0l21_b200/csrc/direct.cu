@@ -311,6 +311,10 @@ __global__ __launch_bounds__(256) void peel_coop_kernel(PeelArgs A) {
     const unsigned __int128 t128 = ((unsigned __int128)A.m << level) / n;
     const uint64_t thr = t128 > 0xFFFFFFFFull ? 0xFFFFFFFFull : (uint64_t)t128;
     unsigned *cinit = A.ctr + (level & 1);
+    // next level's init counter: idle now (last read as this level's predecessor's nf,
+    // which every thread did before a grid.sync, or which was 0), and first appended to
+    // after the grid.sync below, so the barrier orders this reset before its next use
+    if (gtid == 0) A.ctr[(level + 1) & 1] = 0;
     // frontier formation (Algorithm 1 line 4-6)
     for (uint64_t base = gtid & ~31ull; base < n; base += gthreads) {
       const uint64_t v = base + lane;
@@ -319,7 +323,6 @@ __global__ __launch_bounds__(256) void peel_coop_kernel(PeelArgs A) {
     }
     grid.sync();
     unsigned nf = *cinit;
-    if (gtid == 0) A.ctr[(level + 1) & 1] = 0;  // next level's init counter
     while (nf > 0) {
       unsigned *cnext = A.ctr + 2 + (r & 1);
       // mark + split by degree

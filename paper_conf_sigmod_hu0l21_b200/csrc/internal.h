@@ -86,7 +86,15 @@ uint32_t device_max_u32(const uint32_t *a, uint64_t n, cudaStream_t s);
 void direct_graph(Graph &g, int rule);
 void ensure_od(Graph &g);  // out-degrees d~ (original ids), max d~, Eq.1 numerator
 // reorder.cu
-void reorder_graph(Graph &g, int rule, const tc_aorder_params &p);
+// A-order permutation source: by default the host greedy runs here; tc_reorder_dist runs it
+// on rank 0 only and broadcasts pi / bucket_off (AOrderSource filled by api.cu)
+struct AOrderSource {
+  // produce g.perm (device, n), g.bucket_off (device), g.h_bucket_off, g.eq3 from the
+  // host out-degrees; returns false to fall back to the local host greedy
+  virtual bool produce(Graph &g, const std::vector<uint32_t> &h_od, const tc_aorder_params &p) = 0;
+  virtual ~AOrderSource() {}
+};
+void reorder_graph(Graph &g, int rule, const tc_aorder_params &p, AOrderSource *src = nullptr);
 void build_oriented_csr(Graph &g);
 // aorder.cpp (host, Algorithm 2)
 void aorder_host(const std::vector<uint32_t> &od, const tc_aorder_params &p, std::vector<uint32_t> &perm,
@@ -95,8 +103,11 @@ void aorder_units(const std::vector<int64_t> &S, const std::vector<uint8_t> &act
                   std::vector<uint32_t> &pos, std::vector<uint32_t> &bucket_off, int64_t &eq3);
 std::vector<int64_t> superiority_table(uint32_t maxd, const tc_aorder_params &p);
 // count.cu
+// d_T: optional device accumulator (zeroed by the caller): the count is added there and not
+// read back (returns 0), so a collective can consume it on the stream (tc_count_dist)
 uint64_t count_graph(Graph &g, uint32_t u_begin, uint32_t u_end, uint64_t *d_tv /*new labels or null*/,
-                     float *kernel_ms, uint64_t *launches, int mode = -1 /*-1: 1 if d_tv else 0; 2 = per-edge*/);
+                     float *kernel_ms, uint64_t *launches, int mode = -1 /*-1: 1 if d_tv else 0; 2 = per-edge*/,
+                     unsigned long long *d_T = nullptr);
 // per-edge support in CSR positions (final labels) -> canonical order of g.edges (original ids)
 void map_edges_canonical(Graph &g, const uint64_t *d_te, uint64_t *d_out);
 void gather_per_vertex(Graph &g, const uint64_t *d_tnew, uint64_t *d_out);

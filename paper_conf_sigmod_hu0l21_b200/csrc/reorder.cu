@@ -218,7 +218,7 @@ void build_oriented_csr(Graph &g) {
   g.units_ready = false;
 }
 
-void reorder_graph(Graph &g, int rule, const tc_aorder_params &p) {
+void reorder_graph(Graph &g, int rule, const tc_aorder_params &p, AOrderSource *src) {
   cudaStream_t s = g.stream;
   const uint32_t n = g.n;
   if (rule != TC_REORDER_NONE) ensure_od(g);  // D-order / A-order read d~
@@ -245,6 +245,13 @@ void reorder_graph(Graph &g, int rule, const tc_aorder_params &p) {
     std::vector<uint32_t> h_od(n), h_perm;
     if (n) TC_CUDA(cudaMemcpyAsync(h_od.data(), g.od.get(), sizeof(uint32_t) * n, cudaMemcpyDeviceToHost, s));
     TC_CUDA(cudaStreamSynchronize(s));
+    if (src && src->produce(g, h_od, p)) {
+      g.identity_perm = n == 0;
+      g.reorder_rule = rule;
+      build_oriented_csr(g);
+      g.state = G_ORDERED;
+      return;
+    }
     aorder_host(h_od, p, h_perm, g.h_bucket_off, g.eq3);
     if (n) {
       g.perm.alloc(n, s);

@@ -424,8 +424,8 @@ def test_bitmap_intersection():
 @pytest.mark.parametrize("d,r", [("degree", "none"), ("paper", "paper"), ("id", "degree")])
 def test_edge_aorder_schedule(d, r):
     """Schedule "edge_aorder": the units and buckets equal the oracle's Algorithm 2 over the
-    per-edge work items (same superiorities, same greedy), and every count mode gives the
-    oracle's T / t(v) / support on every slice."""
+    edge units (same superiorities, same greedy), and every count mode gives the oracle's
+    T / t(v) / support on every slice."""
     for seed, (sc, ef) in enumerate(((10, 8), (12, 16))):
         spec = graphgen.rmat_spec(sc, ef, 300 + seed)
         src, dst = graphgen.generate_cpu(spec)
@@ -433,7 +433,7 @@ def test_edge_aorder_schedule(d, r):
             ref = oracle.run(src, dst, spec.n, d, r, per_vertex=True, k=k, order=order)
             g = tc.Graph(src, dst, spec.n).direct(d).reorder(r, k=k, order=order).set_schedule("edge_aorder")
             try:
-                units, uoff = g.export_units(k=k)
+                units, uoff = g.export_units()
                 want_u, want_off = oracle.edge_units(ref["offs"], ref["col"], k=k, order=order)
                 assert np.array_equal(units, want_u) and np.array_equal(uoff, want_off)
                 assert g.stats()["eq3_units"] >= 0
@@ -444,6 +444,7 @@ def test_edge_aorder_schedule(d, r):
                 assert sum(g.count_range(a, b) for a, b in zip(bounds, bounds[1:])) == ref["T"]
                 T, te = g.count_edges()
                 assert T == ref["T"] and int(te.sum()) == 3 * T
+                assert np.array_equal(te, oracle.edge_support(ref["edges"], spec.n))
             finally:
                 g.free()
     for name in ("K12", "W9", "B10", "petersen"):

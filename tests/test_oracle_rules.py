@@ -7,6 +7,7 @@ are pinned by hand-traced cases (tests/golden/) and by the invariants the paper
 states (Lemma 4.1, acyclicity P:220, Eq.11 bound P:319-323)."""
 import itertools
 import math
+import os
 
 import numpy as np
 import pytest
@@ -14,7 +15,7 @@ import pytest
 import graphgen
 import oracle
 from tests import graphs
-from tests.conftest import read_golden
+from tests.conftest import GOLDEN, read_golden
 
 
 def _edge_dirs(res_edges, dirs):
@@ -154,6 +155,33 @@ def test_aorder_golden():
     assert perm.tolist() == g["perm_lpt"] and boff.tolist() == g["bucket_off_lpt"]
     perm, _ = oracle.reorder(od, "degree")
     assert perm.tolist() == g["perm_dorder"]
+    # hand-computed superiorities and Eq.3 objectives
+    assert [oracle.superiority(int(d)) if d else 0 for d in od] == g["S"]
+    for order, key in ((0, "eq3"), (1, "eq3_lpt")):
+        perm, boff = oracle.reorder(od, "paper", k=g["k"], order=order)
+        assert oracle.objective_eq3(boff, perm, od) == g[key]
+
+
+def read_superiority_golden():
+    rows = []
+    with open(os.path.join(GOLDEN, "superiority_hand.txt")) as f:
+        for line in f:
+            line = line.split("#", 1)[0].split()
+            if not line:
+                continue
+            assert line[0] == "sup"
+            d, lam, alpha, beta, S, bw = line[1:]
+            bw = None if bw == "-" else [float(x) for x in bw.split(",")]
+            rows.append((int(d), float(lam), float(alpha), float(beta), int(S), bw))
+    return rows
+
+
+def test_superiority_golden():
+    """S(d) with a BW table and alpha, beta != 1/2, worked by hand (Eq.19-20, Q15, Q20)."""
+    rows = read_superiority_golden()
+    assert len(rows) >= 10
+    for d, lam, alpha, beta, S, bw in rows:
+        assert oracle.superiority(d, lam=lam, alpha=alpha, beta=beta, bw=bw) == S, (d, lam, alpha, beta, bw)
 
 
 @pytest.mark.parametrize("k", [1, 3, 8, 32, 128])
@@ -281,8 +309,8 @@ def test_aorder_units_equal_superiority_round_robin():
         assert list(boff) == [j * k for j in range(b + 1)]
 
 
-def test_edge_units_cover_every_wedge_item():
-    """Edge units of a CSR: every (u, 32-edge chunk) with a wedge appears once."""
+def test_edge_units_cover_every_edge_with_work():
+    """Edge units of a CSR: every directed edge u->v with d~(v) >= 1 appears once."""
     src, dst = graphgen.generate_cpu(graphgen.rmat_spec(9, 8, 31))
     res = oracle.run(src, dst, 1 << 9, "degree", "none")
     offs, col = res["offs"].astype(np.int64), res["col"]
@@ -290,8 +318,51 @@ def test_edge_units_cover_every_wedge_item():
     od = np.diff(offs)
     want = set()
     for u in range(len(od)):
-        for c0 in range(0, int(od[u]) if od[u] >= 2 else 0, 32):
-            if (od[col[offs[u] + c0: offs[u] + min(od[u], c0 + 32)]] > 0).any():
-                want.add((u << 32) | c0)
+        for j in range(int(od[u])):
+            if od[col[offs[u] + j]] > 0:
+                want.add((u << 32) | j)
     assert sorted(units.tolist()) == sorted(want) and len(units) == len(want)
     assert boff[-1] == len(units)
+
+
+def test_edge_units_golden():
+    """Hand-traced edge-unit A-order (tests/golden/edge_units_hand7.txt)."""
+    g = read_golden("edge_units_hand7.txt")
+    offs, col = np.array(g["offs"], np.int64), np.array(g["col"], np.uint32)
+    lam = g["lambda_milli"] / 1000.0
+    S, act = oracle.edge_unit_superiority(offs, col, lam=lam)
+    assert S.tolist() == g["S"] and act.tolist() == g["active"]
+    units, boff = oracle.edge_units(offs, col, k=g["k"], lam=lam)
+    assert [int(x) >> 32 for x in units] == g["unit_u"]
+    assert [int(x) & 0xFFFFFFFF for x in units] == g["unit_j"]
+    assert boff.tolist() == g["bucket_off"]
+    # Eq.3 over the unit buckets
+    pos = {int(x): i for i, x in enumerate(units)}
+    src = np.repeat(np.arange(len(offs) - 1), np.diff(offs))
+    per_unit = {(int(src[p]) << 32) | int(p - offs[src[p]]): int(S[p]) for p in range(len(S)) if act[p]}
+    eq3 = sum(abs(sum(per_unit[int(units[i])] for i in range(boff[b], boff[b + 1])))
+              for b in range(len(boff) - 1))
+    assert eq3 == g["eq3"] and len(pos) == len(units)
+
+
+@pytest.mark.parametrize("seed", [0, 1, 2])
+def test_oriented_csr_by_definition(seed):
+    """The oriented, relabelled CSR holds exactly the directed edges (pi(s), pi(t)), each
+    out-list ascending; the one-call O1 (qsort) equals the library-sort O1."""
+    rng = np.random.default_rng(seed)
+    n = 300
+    src = rng.integers(0, n, 4000).astype(np.uint32)
+    dst = rng.integers(0, n, 4000).astype(np.uint32)
+    e = oracle.simple_graph(src, dst, n)
+    buf = np.zeros(len(src), np.uint64)
+    m1 = oracle.lib().orc_simple_graph(oracle._p(src), oracle._p(dst), len(src), n, oracle._p(buf))
+    assert np.array_equal(buf[:m1], e)
+    dirs, _ = oracle.direct(e, n, "degree")
+    perm = rng.permutation(n).astype(np.uint32)
+    offs, col = oracle.oriented_csr(e, n, dirs, perm)
+    want = {}
+    for (fr, to) in _edge_dirs(e, dirs):
+        want.setdefault(int(perm[fr]), []).append(int(perm[to]))
+    for x in range(n):
+        assert col[offs[x]:offs[x + 1]].tolist() == sorted(want.get(x, []))
+    assert offs[-1] == len(e)
