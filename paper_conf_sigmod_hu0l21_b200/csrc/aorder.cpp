@@ -19,6 +19,7 @@
 #include <algorithm>
 #include <cmath>
 #include <cstdint>
+#include <mutex>
 #include <stdexcept>
 #include <thread>
 #include <vector>
@@ -213,6 +214,13 @@ struct MonoQueue {
     refill();
   }
   bool empty() const { return rpos == run.size() && heap.empty(); }
+  template <class F>
+  void for_each(F f) const {  // every key still in the queue
+    for (size_t i = rpos; i < run.size(); ++i) f(run[i]);
+    for (uint64_t x : heap) f(x);
+    for (size_t b = cur + 1; b < bins.size(); ++b)
+      for (uint64_t x : bins[b]) f(x);
+  }
   uint64_t top() const {
     const uint64_t a = rpos < run.size() ? run[rpos] : UINT64_MAX;
     const uint64_t b = heap.empty() ? UINT64_MAX : heap[0];
@@ -259,35 +267,83 @@ static unsigned host_threads(size_t n) {
   return std::max(1u, std::min(h ? h : 1u, 32u));
 }
 
+// Host workspace of the greedy, kept across calls (grow-only; first-touch page faults of
+// ~10 B per unit otherwise cost as much as the greedy itself).  One A-order at a time.
+struct AOrderWorkspace {
+  std::mutex mu;
+  std::vector<uint32_t> vmem, vcomp, bucket_of, rank_of;
+  std::vector<int64_t> smem, scomp;  // S of vmem[i] / vcomp[i]
+};
+static AOrderWorkspace &workspace() {
+  static AOrderWorkspace w;
+  return w;
+}
+template <class T>
+static T *grow(std::vector<T> &v, size_t n) {
+  if (v.size() < n) v.resize(n);
+  return v.data();
+}
+
 template <class SF, class AF>
-static void aorder_core(size_t n, SF S, AF active, uint32_t k, int order, std::vector<uint32_t> &perm,
+static void aorder_core(size_t n, SF S, AF active, uint32_t k, int order, uint32_t *perm,
                         std::vector<uint32_t> &bucket_off, int64_t &eq3) {
-  // line 3-4: V_mem / V_comp in ascending unit index (per-chunk counts, then placement)
+  AOrderWorkspace &W = workspace();
+  std::lock_guard<std::mutex> lock(W.mu);
+  // line 3-4: V_mem / V_comp in ascending unit index: per-chunk counts (with max |S| and
+  // the least nonzero |S| of each class, for the queue's key packing), then placement of
+  // each unit and its S, all on the host cores
   const unsigned T = host_threads(n);
   std::vector<size_t> cm(T + 1, 0), cc(T + 1, 0), ci(T + 1, 0);
+  std::vector<int64_t> tmax(T, 0), tmin1(T, INT64_MAX), tmin2(T, INT64_MAX);
   par_chunks(n, T, [&](size_t lo, size_t hi, unsigned t) {
     size_t a = 0, c = 0, z = 0;
+    int64_t mx = 0, m1 = INT64_MAX, m2 = INT64_MAX;
     for (size_t v = lo; v < hi; ++v) {
-      if (!active(v)) ++z;
-      else if (S(v) > 0) ++a;
-      else ++c;
+      if (!active(v)) {
+        ++z;
+        continue;
+      }
+      const int64_t sv = S(v), av = std::llabs(sv);
+      mx = std::max(mx, av);
+      if (sv > 0) {
+        ++a;
+        m1 = std::min(m1, av);
+      } else {
+        ++c;
+        if (av) m2 = std::min(m2, av);
+      }
     }
     cm[t + 1] = a;
     cc[t + 1] = c;
     ci[t + 1] = z;
+    tmax[t] = mx;
+    tmin1[t] = m1;
+    tmin2[t] = m2;
   });
+  int64_t smax = 0, smin1 = INT64_MAX, smin2 = INT64_MAX;  // max |S|; min nonzero |S| per phase
   for (unsigned t = 0; t < T; ++t) {
     cm[t + 1] += cm[t];
     cc[t + 1] += cc[t];
     ci[t + 1] += ci[t];
+    smax = std::max(smax, tmax[t]);
+    smin1 = std::min(smin1, tmin1[t]);
+    smin2 = std::min(smin2, tmin2[t]);
   }
-  std::vector<uint32_t> vmem(cm[T]), vcomp(cc[T]);
+  const size_t nmem = cm[T], ncomp = cc[T];
+  uint32_t *vmem = grow(W.vmem, nmem), *vcomp = grow(W.vcomp, ncomp);
+  int64_t *smem = grow(W.smem, nmem), *scomp = grow(W.scomp, ncomp);
   par_chunks(n, T, [&](size_t lo, size_t hi, unsigned t) {
     size_t a = cm[t], c = cc[t];
     for (size_t v = lo; v < hi; ++v) {
       if (!active(v)) continue;
-      if (S(v) > 0) vmem[a++] = (uint32_t)v;
-      else vcomp[c++] = (uint32_t)v;
+      const int64_t sv = S(v);
+      if (sv > 0) {
+        smem[a] = sv;
+        vmem[a++] = (uint32_t)v;
+      } else {
+        scomp[c] = sv;
+        vcomp[c++] = (uint32_t)v;
+      }
     }
   });
   if (order == 1) {  // LPT option (Q18): descending |S|, ties by index
@@ -295,101 +351,95 @@ static void aorder_core(size_t n, SF S, AF active, uint32_t k, int order, std::v
       int64_t x = std::llabs(S(a)), y = std::llabs(S(b));
       return x != y ? x > y : a < b;
     };
-    std::sort(vmem.begin(), vmem.end(), lpt);
-    std::sort(vcomp.begin(), vcomp.end(), lpt);
+    std::sort(vmem, vmem + nmem, lpt);
+    std::sort(vcomp, vcomp + ncomp, lpt);
+    for (size_t i = 0; i < nmem; ++i) smem[i] = S(vmem[i]);
+    for (size_t i = 0; i < ncomp; ++i) scomp[i] = S(vcomp[i]);
   }
-  const size_t nact = vmem.size() + vcomp.size();
+  const size_t nact = nmem + ncomp;
   const size_t b = (nact + k - 1) / k;
   std::vector<int64_t> mem_sup(b, 0);        // line 1
   std::vector<uint32_t> fill(b, 0);
-  std::vector<uint32_t> bucket_of(n), rank_of(n);  // insertion record: bucket, rank in it
-  std::vector<uint8_t> alive(b, 1);
-  // Phase 1 / phase 2 priority queues.  Packed 4-ary tree when max|mem_sup| and the bucket
-  // index fit 63 bits (always for the default parameters), else the generic tree.
-  int64_t smax = 0, smin1 = INT64_MAX, smin2 = INT64_MAX;  // max |S|; min nonzero |S| per phase
-  for (uint32_t v : vmem) {
-    int64_t a = std::llabs(S(v));
-    smax = std::max(smax, a);
-    if (a) smin1 = std::min(smin1, a);
-  }
-  for (uint32_t v : vcomp) {
-    int64_t a = std::llabs(S(v));
-    smax = std::max(smax, a);
-    if (a) smin2 = std::min(smin2, a);
-  }
+  uint32_t *bucket_of = grow(W.bucket_of, n), *rank_of = grow(W.rank_of, n);  // insertion record
   const int ib = b > 1 ? 64 - __builtin_clzll((unsigned long long)(b - 1)) : 1;
   const long double bound = (long double)smax * (long double)k * 2.0L + 2.0L;  // |mem_sup| < k smax
   const bool packed = bound * (long double)(1ull << ib) < 9.0e18L;
-  auto run = [&](auto &q) {
-    q.want_max = false;                      // line 2: min queue
+  if (b && packed) {
+    // Packed keys ((±mem_sup + off) << ib) | index: a bucket's mem_sup lives only in its key
+    // (the popped key plus S << ib is the updated key), so a placement touches the queue,
+    // the bucket's fill count and sequential per-unit arrays only.
+    const int64_t off = (int64_t)(smax * (int64_t)k + 1);
+    const uint64_t imask = (1ull << ib) - 1;
+    const uint64_t max_pk = ((uint64_t)(2 * off) << ib) | imask;
+    auto pack = [&](size_t i, int64_t sup, bool want_max) {
+      return ((uint64_t)((want_max ? -sup : sup) + off) << ib) | (uint64_t)i;
+    };
+    MonoQueue q;
+    std::vector<uint64_t> keys;
+    keys.reserve(b);
+    for (size_t i = 0; i < b; ++i) keys.push_back(pack(i, 0, false));
+    q.build(keys, max_pk, smin1 == INT64_MAX ? 0 : (uint64_t)smin1 << ib);  // line 2: min queue
+    for (size_t i = 0; i < nmem; ++i) {          // line 5
+      const uint64_t pk = q.top();
+      const size_t bk = (size_t)(pk & imask);    // line 6
+      const uint32_t r = fill[bk]++;
+      bucket_of[vmem[i]] = (uint32_t)bk;        // line 7
+      rank_of[vmem[i]] = r;
+      const uint64_t npk = pk + ((uint64_t)smem[i] << ib);  // line 8: mem_sup += S(v)
+      const bool live = r + 1 < k;
+      if (!live) mem_sup[bk] = (int64_t)(npk >> ib) - off;
+      q.replace_top(npk, live);                  // line 9
+    }
+    q.for_each([&](uint64_t pk) { mem_sup[pk & imask] = (int64_t)(pk >> ib) - off; });
+    keys.clear();
+    for (size_t i = 0; i < b; ++i)
+      if (fill[i] < k) keys.push_back(pack(i, mem_sup[i], true));
+    q.build(keys, max_pk, smin2 == INT64_MAX ? 0 : (uint64_t)smin2 << ib);  // line 10: max queue
+    for (size_t i = 0; i < ncomp; ++i) {         // line 11
+      const uint64_t pk = q.top();
+      const size_t bk = (size_t)(pk & imask);    // line 12
+      const uint32_t r = fill[bk]++;
+      bucket_of[vcomp[i]] = (uint32_t)bk;       // line 13
+      rank_of[vcomp[i]] = r;
+      const uint64_t npk = pk + ((uint64_t)(-scomp[i]) << ib);  // line 14: mem_sup += S(v) <= 0
+      const bool live = r + 1 < k;
+      if (!live) mem_sup[bk] = off - (int64_t)(npk >> ib);
+      q.replace_top(npk, live);                  // line 15
+    }
+    q.for_each([&](uint64_t pk) { mem_sup[pk & imask] = off - (int64_t)(pk >> ib); });
+  } else if (b) {
+    // generic tournament tree (mem_sup beyond the packed range)
+    std::vector<uint8_t> alive(b, 1);
+    Tournament q;
+    q.want_max = false;                          // line 2: min queue
     q.build(b, mem_sup, alive);
-    for (uint32_t v : vmem) {                // line 5
-      int64_t bk = q.top();                  // line 6
-      bucket_of[v] = (uint32_t)bk;          // line 7
-      rank_of[v] = fill[bk]++;
-      mem_sup[bk] += S(v);               // line 8
+    for (size_t i = 0; i < nmem; ++i) {          // line 5
+      const int64_t bk = q.top();                // line 6
+      bucket_of[vmem[i]] = (uint32_t)bk;        // line 7
+      rank_of[vmem[i]] = fill[bk]++;
+      mem_sup[bk] += smem[i];                    // line 8
       if (fill[bk] == k) alive[bk] = 0;
       q.update((size_t)bk, mem_sup[bk], alive[bk]);  // line 9
     }
-    q.want_max = true;                       // line 10: max queue
+    q.want_max = true;                           // line 10: max queue
     q.build(b, mem_sup, alive);
-    for (uint32_t v : vcomp) {               // line 11
-      int64_t bk = q.top();                  // line 12
-      bucket_of[v] = (uint32_t)bk;          // line 13
-      rank_of[v] = fill[bk]++;
-      mem_sup[bk] += S(v);               // line 14
+    for (size_t i = 0; i < ncomp; ++i) {         // line 11
+      const int64_t bk = q.top();                // line 12
+      bucket_of[vcomp[i]] = (uint32_t)bk;       // line 13
+      rank_of[vcomp[i]] = fill[bk]++;
+      mem_sup[bk] += scomp[i];                   // line 14
       if (fill[bk] == k) alive[bk] = 0;
       q.update((size_t)bk, mem_sup[bk], alive[bk]);  // line 15
     }
-  };
-  if (b) {
-    if (packed) {
-      const int64_t off = (int64_t)(smax * (int64_t)k + 1);
-      const uint64_t imask = (1ull << ib) - 1;
-      const uint64_t max_pk = ((uint64_t)(2 * off) << ib) | imask;
-      auto pack = [&](size_t i, int64_t sup, bool want_max) {
-        return ((uint64_t)((want_max ? -sup : sup) + off) << ib) | (uint64_t)i;
-      };
-      MonoQueue q;
-      std::vector<uint64_t> keys;
-      keys.reserve(b);
-      for (size_t i = 0; i < b; ++i) keys.push_back(pack(i, 0, false));
-      q.build(keys, max_pk, smin1 == INT64_MAX ? 0 : (uint64_t)smin1 << ib);  // line 2: min queue
-      for (uint32_t v : vmem) {              // line 5
-        const size_t bk = (size_t)(q.top() & imask);  // line 6
-        bucket_of[v] = (uint32_t)bk;        // line 7
-        rank_of[v] = fill[bk]++;
-        mem_sup[bk] += S(v);             // line 8
-        if (fill[bk] == k) alive[bk] = 0;
-        q.replace_top(pack(bk, mem_sup[bk], false), alive[bk]);  // line 9
-      }
-      keys.clear();
-      for (size_t i = 0; i < b; ++i)
-        if (alive[i]) keys.push_back(pack(i, mem_sup[i], true));
-      q.build(keys, max_pk, smin2 == INT64_MAX ? 0 : (uint64_t)smin2 << ib);  // line 10: max queue
-      for (uint32_t v : vcomp) {             // line 11
-        const size_t bk = (size_t)(q.top() & imask);  // line 12
-        bucket_of[v] = (uint32_t)bk;        // line 13
-        rank_of[v] = fill[bk]++;
-        mem_sup[bk] += S(v);             // line 14
-        if (fill[bk] == k) alive[bk] = 0;
-        q.replace_top(pack(bk, mem_sup[bk], true), alive[bk]);  // line 15
-      }
-    } else {
-      Tournament q;
-      run(q);
-    }
   }
-  // line 16-20: buckets in index order, members in insertion order (a stable counting
-  // sort of the insertion record: phase-1 vertices first, each phase in iteration order)
-  perm.assign(n, 0);
+  // line 16-20: buckets in index order, members in insertion order (bucket start + rank);
+  // inactive units last in unit order (Q16)
   bucket_off.assign(b + 1, 0);
   eq3 = 0;
   for (size_t i = 0; i < b; ++i) {
     bucket_off[i + 1] = bucket_off[i] + fill[i];
     eq3 += std::llabs(mem_sup[i]);           // Eq.3 objective (λ folded into S)
   }
-  // members in insertion order (bucket start + rank); inactive units last in unit order (Q16)
   const uint32_t inactive0 = bucket_off[b];
   par_chunks(n, T, [&](size_t lo, size_t hi, unsigned t) {
     uint32_t idx = inactive0 + (uint32_t)ci[t];
@@ -400,25 +450,23 @@ static void aorder_core(size_t n, SF S, AF active, uint32_t k, int order, std::v
 
 void aorder_units(const std::vector<int64_t> &Sv, const std::vector<uint8_t> &act, uint32_t k, int order,
                   std::vector<uint32_t> &perm, std::vector<uint32_t> &bucket_off, int64_t &eq3) {
+  perm.resize(Sv.size());
   aorder_core(
-      Sv.size(), [&](size_t v) -> int64_t { return Sv[v]; }, [&](size_t v) { return act[v] != 0; }, k, order, perm,
-      bucket_off, eq3);
+      Sv.size(), [&](size_t v) -> int64_t { return Sv[v]; }, [&](size_t v) { return act[v] != 0; }, k, order,
+      perm.data(), bucket_off, eq3);
 }
 
-void aorder_host(const std::vector<uint32_t> &od, const tc_aorder_params &p, std::vector<uint32_t> &perm,
+void aorder_host(const uint32_t *od, size_t n, const tc_aorder_params &p, uint32_t *perm,
                  std::vector<uint32_t> &bucket_off, int64_t &eq3) {
-  const size_t n = od.size();
   uint32_t maxd = 0;
-  for (uint32_t d : od) maxd = std::max(maxd, d);
-  // superiority per degree value: a table over the degrees present when the range is modest
+  for (size_t v = 0; v < n; ++v) maxd = std::max(maxd, od[v]);
+  // superiority per degree value: a table over the degrees up to max d~ when the range is
+  // modest (S is evaluated once per degree value, Q20)
   const bool use_table = maxd <= (1u << 24);
   std::vector<int64_t> table;
   if (use_table) {
     table.assign((size_t)maxd + 1, 0);
-    std::vector<uint8_t> seen((size_t)maxd + 1, 0);
-    for (uint32_t d : od) seen[d] = 1;
-    for (uint32_t d = 1; d <= maxd; ++d)
-      if (seen[d]) table[d] = memory_superiority(d, p);
+    for (uint32_t d = 1; d <= maxd; ++d) table[d] = memory_superiority(d, p);
   }
   // d~ = 0: no work, F_c(0) undefined (Q16) -> not active
   aorder_core(

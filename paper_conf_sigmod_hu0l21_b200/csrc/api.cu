@@ -293,14 +293,13 @@ namespace {
 struct BroadcastAOrder : AOrderSource {
   nccl::Comm_t comm;
   int rank, root = 0;
-  bool produce(Graph &g, const std::vector<uint32_t> &h_od, const tc_aorder_params &p) override {
+  bool produce(Graph &g, const uint32_t *h_od, uint32_t *h_perm, const tc_aorder_params &p) override {
     nccl::Api &a = nccl::api();
     cudaStream_t s = g.stream;
     const uint32_t n = g.n;
-    std::vector<uint32_t> h_perm;
     uint64_t hdr[2] = {0, 0};
     if (rank == root) {
-      aorder_host(h_od, p, h_perm, g.h_bucket_off, g.eq3);
+      aorder_host(h_od, n, p, h_perm, g.h_bucket_off, g.eq3);
       hdr[0] = g.h_bucket_off.size();
       hdr[1] = (uint64_t)g.eq3;
     }
@@ -319,7 +318,7 @@ struct BroadcastAOrder : AOrderSource {
     if (n) g.perm.alloc(n, s);
     g.bucket_off.alloc(nb1, s);
     if (rank == root) {
-      if (n) TC_CUDA(cudaMemcpyAsync(g.perm.get(), h_perm.data(), sizeof(uint32_t) * n, cudaMemcpyHostToDevice, s));
+      if (n) TC_CUDA(cudaMemcpyAsync(g.perm.get(), h_perm, sizeof(uint32_t) * n, cudaMemcpyHostToDevice, s));
       TC_CUDA(cudaMemcpyAsync(g.bucket_off.get(), g.h_bucket_off.data(), sizeof(uint32_t) * nb1,
                               cudaMemcpyHostToDevice, s));
     }

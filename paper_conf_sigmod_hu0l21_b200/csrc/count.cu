@@ -23,6 +23,7 @@
 #include <map>
 #include <mutex>
 #include <tuple>
+#include <type_traits>
 #include <vector>
 
 #include "internal.h"
@@ -169,19 +170,22 @@ struct Pow2Search {  // full fixed-depth binary search over the +inf-padded slic
     return lds32(p) == w;
   }
 };
-// Bracketed binary search: a per-item table maps the value bucket (w - lo) >> sh to the
-// first list position of that bucket; the binary search then only spans the bucket
-// (S2 = ceil(log2 max bucket occupancy) steps instead of ceil(log2 d~(u))).  Elements
-// past the bucket are larger than w (buckets are monotone), and the slice carries +inf
-// padding past its end, so no bounds checks are needed.
-// A w outside [lo, hi] maps to bucket B (clamped), whose entry is L: the probes then read
-// the +inf padding (2^S2 - 1 < 64 entries past L) and end on an element != w.
-template <int S2>
+// Bracketed binary search: a per-item table maps the value bucket of w to the first list
+// position of that bucket (as a byte offset from slice[0]); the binary search then only
+// spans the bucket (S2 = ceil(log2 max bucket occupancy) steps instead of
+// ceil(log2 d~(u))).  Elements past the bucket are larger than w (buckets are monotone),
+// and the slice carries +inf padding past its end, so no bounds checks are needed.
+// Relative table (ABS = false): bucket (w - lo) >> sh over the list's own range [lo, hi]; a
+// w outside it maps to bucket B (clamped), whose entry is L: the probes then read the +inf
+// padding (2^S2 - 1 < 64 entries past L) and end on an element != w.  Absolute table
+// (ABS = true, chosen when the list spans the whole label range at the same bucket width):
+// bucket w >> sh over [0, 2^vbits), every label has an entry, no subtraction or clamp.
+template <int S2, bool ABS>
 struct TabSearch {
   uint32_t sa, ta, lo, sh, B, sbase;  // slice / table byte addresses, table size, PV base
   __device__ __forceinline__ bool operator()(uint32_t w, uint32_t &pos) const {
-    const uint32_t b = min((w - lo) >> sh, B);
-    uint32_t p = sa + 4u * lds16(ta + 2u * b);
+    const uint32_t b = ABS ? (w >> sh) : min((w - lo) >> sh, B);
+    uint32_t p = sa + lds16(ta + 2u * b);
 #pragma unroll
     for (int k = S2 - 1; k >= 0; --k) {
       const uint32_t q = p + (4u << k);
@@ -256,35 +260,81 @@ __device__ __forceinline__ void wedge_block(uint32_t j0, uint32_t last, const ui
   }
 }
 
-// All wedges of one chunk: blocks of 4 steps, then a 2- and a 1-step block for the rest
-// (an ER item has ~5 steps: 4 + 1 slots instead of 8).
+// N consecutive 32-wedge steps that all lie in ONE owner list (warp-uniform): lane l takes
+// wedges base + l + 32k, all valid, read from one pointer with immediate offsets; no owner
+// walk, no tail masking (count modes only).
+template <int N, int MODE, class Search>
+__device__ __forceinline__ void fast_block(const uint32_t *__restrict__ p, const Search &search, uint32_t j0,
+                                           uint32_t &cnt) {
+  uint32_t w[N];
+#pragma unroll
+  for (int k = 0; k < N; ++k) w[k] = ldg_u32(p + 32 * k);
+#pragma unroll
+  for (int k = 0; k < N; ++k) {
+    uint32_t pos;
+    const bool hit = search(w[k], pos);
+    cnt += hit ? 1u : 0u;
+    if (MODE == 3) {  // §5.3 balance-point experiment, as in wedge_block
+      uint32_t acc = 0;
+      const uint32_t wi = (j0 >> 5) + k;
+      const int ne = (int)((((uint64_t)wi + 1) * (uint32_t)g_extra) >> 3) - (int)(((uint64_t)wi * (uint32_t)g_extra) >> 3);
+      for (int e = 0; e < ne; ++e) {
+        uint32_t p2;
+        acc += search(w[k] ^ (uint32_t)(e + 1), p2) ? 1u : 0u;
+      }
+      cnt += acc & g_sink_mask;
+    }
+  }
+}
+
+// All wedges of one chunk in blocks of NB (8 for CTA items), 4, 2 and 1 steps of 32.  The
+// owner of each block's first wedge is tracked warp-uniformly; a block that lies entirely
+// in that owner's list (long N+(v): most wedges of a skewed graph) takes fast_block, the
+// others walk per lane from there (wedge_block).
 template <int MODE, class Search, int NB = 4>
 __device__ __forceinline__ uint32_t wedge_loop(const uint32_t *__restrict__ col, const Search &search, uint32_t sbase,
                                                uint32_t cbase, uint32_t lo, uint32_t hi, uint32_t total,
                                                WarpScratch &ws, unsigned long long *tv, uint64_t ebase) {
+  constexpr bool FAST = MODE == 0 || MODE == 3 || MODE == 4;
   uint32_t cnt = 0;
-  uint32_t o = 0, o_end = ws.pre[0];
-  const uint32_t *ob = col + ws.vb[0];  // element j of the current owner list is ob[j]
+  uint32_t uo = 0, uo_end = ws.pre[0];
+  const uint32_t *uob = col + ws.vb[0];  // element j of the uniform owner's list is uob[j]
   const uint32_t last = total - 1, steps = (total + 31) >> 5, lane = lane_id();
+  auto block = [&](auto nconst, uint32_t st) {
+    constexpr int N = decltype(nconst)::value;
+    const uint32_t base = 32 * st;
+    while (uo_end <= base) {  // warp-uniform
+      const uint32_t b0 = uo_end;
+      ++uo;
+      uo_end = ws.pre[uo];
+      uob = col + ws.vb[uo] - b0;
+    }
+    if (FAST && uo_end >= base + 32 * N) {
+      fast_block<N, MODE>(uob + base + lane, search, base + lane, cnt);
+    } else {
+      uint32_t o = uo, o_end = uo_end;
+      const uint32_t *ob = uob;
+      wedge_block<N, MODE>(base + lane, last, col, search, ws, o, o_end, ob, cnt, sbase, cbase, tv, ebase);
+    }
+  };
   uint32_t st = 0;
   if (NB == 8)  // CTA items (register budget 48): 8 gathers in flight per lane
-    for (; st + 8 <= steps; st += 8)
-      wedge_block<8, MODE>(lane + 32 * st, last, col, search, ws, o, o_end, ob, cnt, sbase, cbase, tv, ebase);
-  for (; st + 4 <= steps; st += 4)
-    wedge_block<4, MODE>(lane + 32 * st, last, col, search, ws, o, o_end, ob, cnt, sbase, cbase, tv, ebase);
+    for (; st + 8 <= steps; st += 8) block(std::integral_constant<int, 8>(), st);
+  for (; st + 4 <= steps; st += 4) block(std::integral_constant<int, 4>(), st);
   if (st + 2 <= steps) {
-    wedge_block<2, MODE>(lane + 32 * st, last, col, search, ws, o, o_end, ob, cnt, sbase, cbase, tv, ebase);
+    block(std::integral_constant<int, 2>(), st);
     st += 2;
   }
-  if (st < steps) wedge_block<1, MODE>(lane + 32 * st, last, col, search, ws, o, o_end, ob, cnt, sbase, cbase, tv, ebase);
+  if (st < steps) block(std::integral_constant<int, 1>(), st);
   (void)lo;
   (void)hi;
   return cnt;
 }
 
 // Builds the bracket table of the staged list s = tc_smem[sbase .. sbase+L) (warp-wide):
-// tab[b] = first index whose bucket (s - lo) >> sh is >= b, b in [0, B]; returns
-// ceil(log2(max bucket occupancy)).
+// tab[b] = 4 * (first index whose bucket (s - lo) >> sh is >= b), b in [0, B] with
+// B = ((hi - lo) >> sh) + 1 (hi >= the list's last element: the absolute table passes
+// lo = 0, hi = 2^vbits - 1); returns ceil(log2(max bucket occupancy)).
 __device__ __forceinline__ int build_bracket(uint32_t sbase, uint32_t tbase, uint32_t L, uint32_t lo, uint32_t hi,
                                              uint32_t sh) {
   const uint32_t B = ((hi - lo) >> sh) + 1;
@@ -292,12 +342,13 @@ __device__ __forceinline__ int build_bracket(uint32_t sbase, uint32_t tbase, uin
   for (uint32_t j = lane_id(); j < L; j += 32) {
     const uint32_t bj = (tc_smem[sbase + j] - lo) >> sh;
     const int bp = j ? (int)((tc_smem[sbase + j - 1] - lo) >> sh) : -1;
-    for (int b = bp + 1; b <= (int)bj; ++b) tab[b] = (uint16_t)j;
+    for (int b = bp + 1; b <= (int)bj; ++b) tab[b] = (uint16_t)(4 * j);
   }
-  if (lane_id() == 0) tab[B] = (uint16_t)L;
+  // buckets past the last element's (absolute tables) and the sentinel B: 4L
+  for (uint32_t b = ((tc_smem[sbase + L - 1] - lo) >> sh) + 1 + lane_id(); b <= B; b += 32) tab[b] = (uint16_t)(4 * L);
   __syncwarp();
   uint32_t mx = 0;
-  for (uint32_t b = lane_id(); b < B; b += 32) mx = max(mx, (uint32_t)tab[b + 1] - tab[b]);
+  for (uint32_t b = lane_id(); b < B; b += 32) mx = max(mx, ((uint32_t)tab[b + 1] - tab[b]) >> 2);
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) mx = max(mx, __shfl_xor_sync(0xffffffffu, mx, o));
   return ceil_log2(mx);
@@ -312,7 +363,8 @@ __device__ __forceinline__ uint32_t warp_chunk(const uint64_t *__restrict__ offs
                                                uint32_t v, bool valid, const uint32_t *list, uint32_t sbase,
                                                uint32_t tbase, uint32_t cbase, uint32_t L, bool padded, uint32_t lo,
                                                uint32_t hi, WarpScratch &ws, unsigned long long *tv, uint32_t vidx,
-                                               uint64_t ua, uint64_t ebase, int S2pre = -1, uint32_t shpre = 0) {
+                                               uint64_t ua, uint64_t ebase, uint32_t vbits, int S2pre = -1,
+                                               uint32_t shpre = 0, int abspre = 0) {
   constexpr bool PV = MODE == 1, PE = MODE == 2;
   const unsigned lane = lane_id();
   uint64_t vb = 0;
@@ -339,10 +391,19 @@ __device__ __forceinline__ uint32_t warp_chunk(const uint64_t *__restrict__ offs
     const int S = padded ? ceil_log2(L) : 0;
     int S2 = S2pre >= 0 ? S2pre : 99;  // S2pre: table prebuilt by the CTA (large kernel)
     uint32_t sh = shpre;
+    bool abs_t = abspre != 0;
+    uint32_t tlo = lo, thi = hi;
     if (MODE != 4 && S2pre < 0 && S >= 6 && tbase != 0xffffffffu && g_bracket && total >= 2 * L) {
       const int span_bits = 32 - __clz(hi - lo);  // bits of (hi - lo)
-      sh = span_bits > S + TS_W ? (uint32_t)(span_bits - S - TS_W) : 0u;
-      S2 = build_bracket(sbase, tbase, L, lo, hi, sh);
+      // a list spanning the whole label range gets the absolute table (same bucket width)
+      abs_t = span_bits >= (int)vbits;
+      const int tb = abs_t ? (int)vbits : span_bits;
+      if (abs_t) {
+        tlo = 0;
+        thi = vbits >= 32 ? 0xffffffffu : (1u << vbits) - 1u;
+      }
+      sh = tb > S + TS_W ? (uint32_t)(tb - S - TS_W) : 0u;
+      S2 = build_bracket(sbase, tbase, L, tlo, thi, sh);
       __syncwarp();
     }
     if (MODE == 4) {  // every staged list has <= 32 entries (host-checked): 1..5 steps only
@@ -354,10 +415,16 @@ __device__ __forceinline__ uint32_t warp_chunk(const uint64_t *__restrict__ offs
       }
     } else if (S2 <= 6) {
       switch (S2) {
-#define TC_TAB(k) \
-  case k:                                                                                                     \
-    cnt = wedge_loop<MODE, TabSearch<k>, NB>(col, TabSearch<k>{smem_addr(sbase), smem_addr(tbase), lo, sh, ((hi - lo) >> sh) + 1, sbase}, \
-                           sbase, cbase, lo, hi, total, ws, tv, ebase);                                       \
+#define TC_TAB(k)                                                                                            \
+  case k:                                                                                                    \
+    if (abs_t)                                                                                               \
+      cnt = wedge_loop<MODE, TabSearch<k, true>, NB>(                                                        \
+          col, TabSearch<k, true>{smem_addr(sbase), smem_addr(tbase), 0u, sh, 0u, sbase}, sbase, cbase, lo, hi, \
+          total, ws, tv, ebase);                                                                             \
+    else                                                                                                     \
+      cnt = wedge_loop<MODE, TabSearch<k, false>, NB>(                                                       \
+          col, TabSearch<k, false>{smem_addr(sbase), smem_addr(tbase), tlo, sh, ((thi - tlo) >> sh) + 1, sbase}, \
+          sbase, cbase, lo, hi, total, ws, tv, ebase);                                                       \
     break;
         TC_TAB(0) TC_TAB(1) TC_TAB(2) TC_TAB(3) TC_TAB(4) TC_TAB(5) TC_TAB(6)
 #undef TC_TAB
@@ -388,7 +455,7 @@ __device__ __forceinline__ uint32_t warp_chunk(const uint64_t *__restrict__ offs
 template <int MODE>
 __device__ __forceinline__ uint64_t warp_item(const uint64_t *__restrict__ offs, const uint32_t *__restrict__ col,
                                               uint32_t u, uint32_t c0, uint32_t sbase, uint32_t cap,
-                                              WarpScratch &ws, unsigned long long *tv) {
+                                              WarpScratch &ws, unsigned long long *tv, uint32_t vbits) {
   constexpr bool PV = MODE == 1, PE = MODE == 2;
   const unsigned lane = lane_id();
   const uint64_t a = offs[u];
@@ -414,7 +481,7 @@ __device__ __forceinline__ uint64_t warp_item(const uint64_t *__restrict__ offs,
   const bool valid = c0 + lane < L;
   const uint32_t v = valid ? list[c0 + lane] : 0u;
   uint32_t cnt = warp_chunk<MODE>(offs, col, v, valid, list, sbase, padded ? sbase + cap + 64 : 0xffffffffu, cbase, L,
-                                  padded, lo, hi, ws, tv, c0 + lane, a, a);
+                                  padded, lo, hi, ws, tv, c0 + lane, a, a, vbits);
   __syncwarp();  // slice reads done before the next item restages it
   if (PV) {
     uint64_t tot = warp_sum((uint64_t)cnt);
@@ -529,7 +596,8 @@ __global__ __launch_bounds__(CT_THREADS, MODE == 4 ? 8 : (MODE == 0 || MODE == 3
                                                                  const uint32_t *__restrict__ col,
                                                                  const uint64_t *__restrict__ items, uint64_t nitems,
                                                                  uint64_t nheavy, unsigned long long *ctr, uint32_t cap,
-                                                                 unsigned long long *T, unsigned long long *tv) {
+                                                                 unsigned long long *T, unsigned long long *tv,
+                                                                 uint32_t vbits) {
   __shared__ WarpScratch s_ws[CT_WARPS];
   const uint32_t slice = warp_id() * warp_stride(cap, MODE == 1 || MODE == 2);
   WarpScratch &ws = s_ws[warp_id()];
@@ -540,7 +608,7 @@ __global__ __launch_bounds__(CT_THREADS, MODE == 4 ? 8 : (MODE == 0 || MODE == 3
     i = __shfl_sync(0xffffffffu, i, 0);
     if (i >= nheavy) break;
     uint64_t it = items[i];
-    acc += warp_item<MODE>(offs, col, (uint32_t)(it >> 32), (uint32_t)it, slice, cap, ws, tv);
+    acc += warp_item<MODE>(offs, col, (uint32_t)(it >> 32), (uint32_t)it, slice, cap, ws, tv, vbits);
   }
   while (true) {  // light items, CHUNK per fetch
     unsigned long long b = 0;
@@ -550,7 +618,7 @@ __global__ __launch_bounds__(CT_THREADS, MODE == 4 ? 8 : (MODE == 0 || MODE == 3
     uint64_t e = min((uint64_t)b + CHUNK, nitems);
     for (uint64_t i = b; i < e; ++i) {
       uint64_t it = items[i];
-      acc += warp_item<MODE>(offs, col, (uint32_t)(it >> 32), (uint32_t)it, slice, cap, ws, tv);
+      acc += warp_item<MODE>(offs, col, (uint32_t)(it >> 32), (uint32_t)it, slice, cap, ws, tv, vbits);
     }
   }
   block_add_u64(acc, T);
@@ -592,7 +660,7 @@ __global__ __launch_bounds__(LG_THREADS, 5) void count_large_kernel(const uint64
                                                                  const uint32_t *__restrict__ col,
                                                                  const uint64_t *__restrict__ items, uint64_t nitems,
                                                                  unsigned long long *ctr, unsigned long long *T,
-                                                                 unsigned long long *tv) {
+                                                                 unsigned long long *tv, uint32_t vbits) {
   uint32_t *s_piece = tc_smem;  // PIECE + 72 words (alignment slack + padding), then the table
   constexpr uint32_t tbase_lg = PIECE + 72;
   __shared__ WarpScratch s_ws[LG_WARPS];
@@ -640,24 +708,30 @@ __global__ __launch_bounds__(LG_THREADS, 5) void count_large_kernel(const uint64
         __syncthreads();
       }
       const uint32_t lo = list[0], hi = list[plen - 1];
-      // CTA-wide bracket table of the piece (shared by all warps of the item)
+      // CTA-wide bracket table of the piece (shared by all warps of the item); absolute
+      // (bucket w >> sh over [0, 2^vbits)) when the piece spans the whole label range
       int S2 = -1;
       uint32_t sh = 0;
+      bool abs_t = false;
       const int S = ceil_log2(plen);
       if (g_bracket && S >= 6) {
         const int span_bits = 32 - __clz(hi - lo);
-        sh = span_bits > S + TS_L ? (uint32_t)(span_bits - S - TS_L) : 0u;
-        const uint32_t B = ((hi - lo) >> sh) + 1;
+        abs_t = span_bits >= (int)vbits;
+        const uint32_t tlo = abs_t ? 0u : lo;
+        const uint32_t thi = abs_t ? (vbits >= 32 ? 0xffffffffu : (1u << vbits) - 1u) : hi;
+        const int tb = abs_t ? (int)vbits : span_bits;
+        sh = tb > S + TS_L ? (uint32_t)(tb - S - TS_L) : 0u;
+        const uint32_t B = ((thi - tlo) >> sh) + 1;
         uint16_t *tab = reinterpret_cast<uint16_t *>(tc_smem + tbase_lg);
         for (uint32_t j = threadIdx.x; j < plen; j += LG_THREADS) {
-          const uint32_t bj = (list[j] - lo) >> sh;
-          const int bp = j ? (int)((list[j - 1] - lo) >> sh) : -1;
-          for (int b = bp + 1; b <= (int)bj; ++b) tab[b] = (uint16_t)j;
+          const uint32_t bj = (list[j] - tlo) >> sh;
+          const int bp = j ? (int)((list[j - 1] - tlo) >> sh) : -1;
+          for (int b = bp + 1; b <= (int)bj; ++b) tab[b] = (uint16_t)(4 * j);
         }
-        if (threadIdx.x == 0) tab[B] = (uint16_t)plen;
+        for (uint32_t b = ((hi - tlo) >> sh) + 1 + threadIdx.x; b <= B; b += LG_THREADS) tab[b] = (uint16_t)(4 * plen);
         __syncthreads();
         uint32_t mx = 0;
-        for (uint32_t b = threadIdx.x; b < B; b += LG_THREADS) mx = max(mx, (uint32_t)tab[b + 1] - tab[b]);
+        for (uint32_t b = threadIdx.x; b < B; b += LG_THREADS) mx = max(mx, ((uint32_t)tab[b + 1] - tab[b]) >> 2);
         mx = warp_max(mx);
         if (lane_id() == 0) s_red[warp_id()] = mx;
         __syncthreads();
@@ -679,7 +753,8 @@ __global__ __launch_bounds__(LG_THREADS, 5) void count_large_kernel(const uint64
         const bool valid = lane_id() < LG_SUB && c0 + lane_id() < cend;
         const uint32_t v = valid ? ldg_u32(col + a + c0 + lane_id()) : 0u;
         cnt += warp_chunk<MODE, MODE == 0 ? 8 : 4>(offs, col, v, valid, list, shift, S2 >= 0 ? tbase_lg : 0xffffffffu, 0xffffffffu, plen,
-                                true, lo, hi, ws, tv, c0 + lane_id(), a, a + p0, S2 >= 0 ? S2 : -2, sh);
+                                true, lo, hi, ws, tv, c0 + lane_id(), a, a + p0, vbits, S2 >= 0 ? S2 : -2, sh,
+                                abs_t ? 1 : 0);
       }
       ucnt += cnt;
       __syncthreads();  // piece fully consumed before the next bulk copy overwrites it
@@ -700,7 +775,8 @@ __global__ __launch_bounds__(CT_THREADS) void count_range_kernel(const uint64_t 
                                                                  const uint32_t *__restrict__ boff, uint32_t kfixed,
                                                                  uint32_t b0, uint32_t nb, uint32_t ub, uint32_t ue,
                                                                  uint32_t cap, unsigned *bucket_ctr,
-                                                                 unsigned long long *T, unsigned long long *tv) {
+                                                                 unsigned long long *T, unsigned long long *tv,
+                                                                 uint32_t vbits) {
   __shared__ WarpScratch s_ws[CT_WARPS];
   __shared__ uint32_t s_bucket;
   const uint32_t slice = warp_id() * warp_stride(cap, MODE == 1 || MODE == 2);
@@ -724,7 +800,7 @@ __global__ __launch_bounds__(CT_THREADS) void count_range_kernel(const uint64_t 
       uint32_t nit = (L + SV - 1) / SV;
       uint32_t first = (warp_id() + CT_WARPS - (t % CT_WARPS)) % CT_WARPS;
       for (uint32_t c = first; c < nit; c += CT_WARPS)
-        acc += warp_item<MODE>(offs, col, (uint32_t)u, c * SV, slice, cap, ws, tv);
+        acc += warp_item<MODE>(offs, col, (uint32_t)u, c * SV, slice, cap, ws, tv, vbits);
       t += nit;
     }
   }
@@ -1091,6 +1167,8 @@ uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *
   } dT{d_T ? d_T : dT_own.get()};
   unsigned long long *tv = reinterpret_cast<unsigned long long *>(d_tv);
   const uint32_t cap = (uint32_t)g_opt_small_cap;
+  // bits of the largest label: absolute bracket tables cover [0, 2^vbits)
+  const uint32_t vbits = g.n > 1 ? 32u - (uint32_t)__builtin_clz(g.n - 1) : 1u;
   int sched = g.schedule;
   // AUTO = BUCKETED for every ordering: measured on B200 (R-MAT s22, profiles/), the
   // dynamic heavy-first item schedule beats the static block-per-bucket model A-order
@@ -1176,7 +1254,7 @@ uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *
         if (kernel_ms) TC_CUDA(cudaEventRecord(e0, s));
         ProfScope prof("count_range", s, 0.0);
         range_fn<<<grid, CT_THREADS, smem, s>>>(g.offs.get(), g.col.get(), boff, k, b0, nb, ub, ue, rcap, bctr.get(),
-                                                dT.get(), tv);
+                                                dT.get(), tv, vbits);
         TC_LAUNCH_CHECK();
         if (kernel_ms) TC_CUDA(cudaEventRecord(e1, s));
         ++nlaunch;
@@ -1232,7 +1310,7 @@ uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *
           unsigned grid = (unsigned)std::min<uint64_t>(nlarge, (uint64_t)num_sms() * occ);
           ProfScope prof("count_large", s, 0.0);
           large_fn<<<grid, LG_THREADS, smem, s>>>(g.offs.get(), g.col.get(), items.get(), nlarge, hist.get() + 64,
-                                                   dT.get(), tv);
+                                                   dT.get(), tv, vbits);
           TC_LAUNCH_CHECK();
           ++nlaunch;
         }
@@ -1254,7 +1332,7 @@ uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *
           unsigned grid = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(want, (uint64_t)num_sms() * occ));
           ProfScope prof("count_small", s, 0.0);
           small_fn<<<grid, CT_THREADS, smem, s>>>(g.offs.get(), g.col.get(), items.get() + nlarge, nsmall, nheavy,
-                                                   hist.get() + 65, cap_small, dT.get(), tv);
+                                                   hist.get() + 65, cap_small, dT.get(), tv, vbits);
           TC_LAUNCH_CHECK();
           ++nlaunch;
         }

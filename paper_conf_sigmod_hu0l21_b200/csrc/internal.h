@@ -2,6 +2,7 @@
 #pragma once
 #include <stdint.h>
 
+#include <mutex>
 #include <vector>
 
 #include "../../include/tc.h"
@@ -91,14 +92,19 @@ void ensure_od(Graph &g);  // out-degrees d~ (original ids), max d~, Eq.1 numera
 struct AOrderSource {
   // produce g.perm (device, n), g.bucket_off (device), g.h_bucket_off, g.eq3 from the
   // host out-degrees; returns false to fall back to the local host greedy
-  virtual bool produce(Graph &g, const std::vector<uint32_t> &h_od, const tc_aorder_params &p) = 0;
+  // h_od[n]: host out-degrees; h_perm[n]: host scratch for pi (both pinned)
+  virtual bool produce(Graph &g, const uint32_t *h_od, uint32_t *h_perm, const tc_aorder_params &p) = 0;
   virtual ~AOrderSource() {}
 };
 void reorder_graph(Graph &g, int rule, const tc_aorder_params &p, AOrderSource *src = nullptr);
 void build_oriented_csr(Graph &g);
 // aorder.cpp (host, Algorithm 2)
-void aorder_host(const std::vector<uint32_t> &od, const tc_aorder_params &p, std::vector<uint32_t> &perm,
+// od[n] -> perm[n] (caller memory, e.g. pinned), bucket_off, Eq.3 objective
+void aorder_host(const uint32_t *od, size_t n, const tc_aorder_params &p, uint32_t *perm,
                  std::vector<uint32_t> &bucket_off, int64_t &eq3);
+// pinned host staging buffers (grow-only; slot 0 / 1), used under g_pinned_mu (reorder.cu)
+uint32_t *pinned_u32(size_t n, int slot);
+extern std::mutex g_pinned_mu;
 void aorder_units(const std::vector<int64_t> &S, const std::vector<uint8_t> &active, uint32_t k, int order,
                   std::vector<uint32_t> &pos, std::vector<uint32_t> &bucket_off, int64_t &eq3);
 std::vector<int64_t> superiority_table(uint32_t maxd, const tc_aorder_params &p);

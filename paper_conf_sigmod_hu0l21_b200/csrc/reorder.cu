@@ -1,3 +1,4 @@
+#include <mutex>
 // reorder.cu — steps a6-a7: vertex ordering and the oriented CSR in the new labels.
 //
 //   NONE    identity ("Original")
@@ -218,6 +219,22 @@ void build_oriented_csr(Graph &g) {
   g.units_ready = false;
 }
 
+// Pinned host staging buffers for the A-order round trip (grow-only; the driver keeps
+// them for the process lifetime).
+std::mutex g_pinned_mu;
+uint32_t *pinned_u32(size_t n, int slot) {
+  static uint32_t *buf[2] = {nullptr, nullptr};
+  static size_t cap[2] = {0, 0};
+  if (cap[slot] < n) {
+    if (buf[slot]) TC_CUDA(cudaFreeHost(buf[slot]));
+    buf[slot] = nullptr;
+    cap[slot] = 0;
+    TC_CUDA(cudaMallocHost((void **)&buf[slot], n * sizeof(uint32_t)));
+    cap[slot] = n;
+  }
+  return buf[slot];
+}
+
 void reorder_graph(Graph &g, int rule, const tc_aorder_params &p, AOrderSource *src) {
   cudaStream_t s = g.stream;
   const uint32_t n = g.n;
@@ -242,26 +259,29 @@ void reorder_graph(Graph &g, int rule, const tc_aorder_params &p, AOrderSource *
     TC_LAUNCH_CHECK();
     g.identity_perm = false;
   } else if (rule == TC_REORDER_PAPER) {
-    std::vector<uint32_t> h_od(n), h_perm;
-    if (n) TC_CUDA(cudaMemcpyAsync(h_od.data(), g.od.get(), sizeof(uint32_t) * n, cudaMemcpyDeviceToHost, s));
+    // d~ down and pi up through pinned staging buffers (kept across calls, one A-order at a
+    // time: the host greedy holds the lock anyway)
+    std::lock_guard<std::mutex> lock(g_pinned_mu);
+    uint32_t *h_od = pinned_u32(n ? n : 1, 0), *h_perm = pinned_u32(n ? n : 1, 1);
+    if (n) TC_CUDA(cudaMemcpyAsync(h_od, g.od.get(), sizeof(uint32_t) * n, cudaMemcpyDeviceToHost, s));
     TC_CUDA(cudaStreamSynchronize(s));
-    if (src && src->produce(g, h_od, p)) {
+    if (src && src->produce(g, h_od, h_perm, p)) {
       g.identity_perm = n == 0;
       g.reorder_rule = rule;
       build_oriented_csr(g);
       g.state = G_ORDERED;
       return;
     }
-    aorder_host(h_od, p, h_perm, g.h_bucket_off, g.eq3);
+    aorder_host(h_od, n, p, h_perm, g.h_bucket_off, g.eq3);
     if (n) {
       g.perm.alloc(n, s);
-      TC_CUDA(cudaMemcpyAsync(g.perm.get(), h_perm.data(), sizeof(uint32_t) * n, cudaMemcpyHostToDevice, s));
+      TC_CUDA(cudaMemcpyAsync(g.perm.get(), h_perm, sizeof(uint32_t) * n, cudaMemcpyHostToDevice, s));
       g.identity_perm = false;
     }
     g.bucket_off.alloc(g.h_bucket_off.size(), s);
     TC_CUDA(cudaMemcpyAsync(g.bucket_off.get(), g.h_bucket_off.data(), sizeof(uint32_t) * g.h_bucket_off.size(),
                             cudaMemcpyHostToDevice, s));
-    TC_CUDA(cudaStreamSynchronize(s));  // host vectors must outlive the copies
+    TC_CUDA(cudaStreamSynchronize(s));  // host buffers must outlive the copies
   }
   g.reorder_rule = rule;
   build_oriented_csr(g);

@@ -20,12 +20,12 @@ int main(int argc, char **argv) {
   fclose(f);
   int reps = argc > 2 ? atoi(argv[2]) : 3;
   tc_aorder_params p{9.682, 0.5, 0.5, nullptr, 0, 32, 0};
-  std::vector<uint32_t> perm, boff;
+  std::vector<uint32_t> perm(n), boff;
   int64_t eq3 = 0;
   uint64_t h = 0;
   for (int r = 0; r < reps; ++r) {
     auto t0 = std::chrono::steady_clock::now();
-    tc::aorder_host(od, p, perm, boff, eq3);
+    tc::aorder_host(od.data(), n, p, perm.data(), boff, eq3);
     auto t1 = std::chrono::steady_clock::now();
     h = 1469598103934665603ull;
     for (uint32_t x : perm) h = (h ^ x) * 1099511628211ull;
