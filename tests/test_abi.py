@@ -37,7 +37,7 @@ def test_binding_mirrors_abi_names():
 
 def test_struct_layouts():
     assert ctypes.sizeof(tc.AOrderParams) == 3 * 8 + 8 + 4 + 4 + 4 + 4  # padded to 8
-    assert ctypes.sizeof(tc.Stats) == 8 * 7 + 8 + 4 * 6 + 8 * 3 + 8 * 5 + 8 + 8 + 8
+    assert ctypes.sizeof(tc.Stats) == 8 * 7 + 8 + 4 * 6 + 8 * 3 + 8 * 5 + 8 + 8 + 8 + 8
 
 
 def test_version_string():
