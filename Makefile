@@ -27,7 +27,7 @@ oracle/liboracle.so: oracle/tc_oracle.c
 # one object per source (parallel make), then one shared library
 TC_OBJS := $(patsubst $(PKG)/csrc/%.cu,build/%.o,$(TC_SRCS)) $(patsubst $(PKG)/csrc/%.cpp,build/%.cpp.o,$(TC_CPP))
 
-build/%.o: $(PKG)/csrc/%.cu $(TC_HDRS) $(PKG)/csrc/internal.h
+build/%.o: $(PKG)/csrc/%.cu $(TC_HDRS) $(PKG)/csrc/internal.h $(PKG)/csrc/count_dev.cuh
 	@mkdir -p build
 	$(NVCC) $(NVFLAGS) -Iinclude -c $< -o $@ 2> build/$*.ptxas.log || (cat build/$*.ptxas.log; false)
 

@@ -219,7 +219,13 @@ tc_status tc_export_units(tc_graph *g, uint64_t *units, uint32_t *unit_off);
  * performs p_c = q/8 extra searches of the staged N+(u) per wedge (whole 32-wedge warp
  * steps, spread evenly), results discarded — the
  * balance-point experiment of §5.3, used to re-fit the A-order model on B200
- * (tools/refit.py); counts are unchanged). */
+ * (tools/refit.py); counts are unchanged), "shorter" (0/1, default 1: in the counts without
+ * per-vertex/per-edge output of the bucketed schedule, every directed edge u->v streams the
+ * SHORTER of N+(u), N+(v) and binary-searches its elements in the other, staged once for
+ * all edges that search it — SURVEY.md §8(a) a9 "the shorter of the two lists per edge ...
+ * probed into the longer list"; 0 = always stream N+(v) against the staged N+(u), Hu's
+ * pattern), "owner_span" / "owner_lspan" (streamed lists per warp / CTA work item of
+ * that schedule, defaults 128 / 2048). */
 tc_status tc_set_option(const char *key, int64_t value);
 
 /* Per-kernel profile since the last reset, as JSON text into buf (host, cap bytes):

@@ -196,6 +196,14 @@ tc_status tc_set_option(const char *key, int64_t value) {
     }
     else if (k == "peel_coop") g_opt_peel_coop = value ? 1 : 0;
     else if (k == "split") g_opt_split = value ? 1 : 0;
+    else if (k == "shorter") g_opt_shorter = value ? 1 : 0;
+    else if (k == "owner_span") {
+      TC_REQUIRE(value >= 32 && value <= (1 << 20) && value % 32 == 0, ST_INVALID, "owner_span: multiple of 32");
+      g_opt_owner_span = (int)value;
+    } else if (k == "owner_lspan") {
+      TC_REQUIRE(value >= 8 && value <= (1 << 24), ST_INVALID, "owner_lspan: 8 .. 2^24");
+      g_opt_owner_lspan = (int)value;
+    }
     else if (k == "small_cap") {
       TC_REQUIRE(value >= 32 && value <= 2048 && (value & (value - 1)) == 0, ST_INVALID,
                  "small_cap must be a power of two in [32, 2048]");

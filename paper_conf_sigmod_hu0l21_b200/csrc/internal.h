@@ -131,5 +131,8 @@ extern int g_opt_extra;  // §5.3 experiment: extra searches per wedge (-1 = pro
 extern int g_opt_intersect;  // 0 binary search, 1 sort-merge (count only)
 extern int g_opt_peel_coop;  // A-direction peel as one cooperative launch
 extern int g_opt_split;  // orientation split CSR build (original labels)
+extern int g_opt_shorter;      // shorter-list owner schedule for count modes
+extern int g_opt_owner_span;   // owners per warp item
+extern int g_opt_owner_lspan;  // owners per CTA item
 
 }  // namespace tc
