@@ -374,8 +374,10 @@ def main():
                 "per_launch_ms": per_launch_ms, "alg_bytes_per_launch": per_launch_bytes}
         if dom == "count":
             roof["kernels"] = [k for k in count_keys if k in prof]
-            roof["bytes_model"] = ("SURVEY.md §8(d) no-reuse 32-B-sector model of the count, computed "
-                                   "exactly per graph by tc_analyze")
+            roof["bytes_model"] = ("SURVEY.md §8(d) no-reuse 32-B-sector model of the count's schedule "
+                                   "(per edge the streamed list = the shorter of N+(u), N+(v), + its "
+                                   "offsets; per source its staged list), computed exactly per graph "
+                                   "by tc_analyze")
 
     line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": t_step, "higher_is_better": True,

@@ -102,7 +102,10 @@ typedef struct {
   uint32_t direct_rule, reorder_rule, schedule;
   uint64_t triangles;            /* last count */
   uint64_t wedges;               /* sum_u sum_{v in N+(u)} d~(v) (after tc_analyze) */
-  uint64_t alg_bytes;            /* count kernel algorithmic DRAM bytes, sector model (tc_analyze) */
+  uint64_t alg_bytes;            /* count kernel algorithmic DRAM bytes, no-reuse 32-B sector model of
+                                    the schedule a plain tc_count runs: per edge the streamed list
+                                    (the shorter one, or N+(v) in Hu's pattern) + its offsets, per
+                                    source its staged list (tc_analyze) */
   double ms_build, ms_direct, ms_reorder, ms_count; /* device time of the last call of each */
   double ms_count_kernel;        /* device time of the count kernels alone (last tc_count) */
   uint64_t count_launches;       /* kernels launched by the last tc_count */

@@ -20,7 +20,8 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libtc_b200.so")
+# TC_B200_LIB: an alternative build of the same library (tools/build_variant.sh experiments)
+LIB_PATH = os.environ.get("TC_B200_LIB") or os.path.join(_HERE, "libtc_b200.so")
 
 TC_OK, TC_ERR_INVALID, TC_ERR_OOM, TC_ERR_CUDA, TC_ERR_NCCL, TC_ERR_STATE = range(6)
 DIRECT = {"id": 0, "degree": 1, "paper": 2}

@@ -17,6 +17,9 @@
 //   F_m = BW(d)^α (Eq.19), F_c = 1/d^β (Eq.20); α = β = 1/2 evaluated literally as
 //   sqrt(BW(d)) and sqrt(1/d) (Eq.22); BW(d) = d unless a table is given (Q15).
 #include <algorithm>
+#include <chrono>
+#include <cstdio>
+#include <cstdlib>
 #include <cmath>
 #include <cstdint>
 #include <mutex>
@@ -284,11 +287,22 @@ static T *grow(std::vector<T> &v, size_t n) {
   return v.data();
 }
 
+// phase timing to stderr when TC_AORDER_TRACE is set (tools/aorder_bench.cpp)
+static bool trace_on() {
+  static const bool on = std::getenv("TC_AORDER_TRACE") != nullptr;
+  return on;
+}
+static double now_ms() {
+  return std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now().time_since_epoch()).count();
+}
+
 template <class SF, class AF>
 static void aorder_core(size_t n, SF S, AF active, uint32_t k, int order, uint32_t *perm,
                         std::vector<uint32_t> &bucket_off, int64_t &eq3) {
   AOrderWorkspace &W = workspace();
   std::lock_guard<std::mutex> lock(W.mu);
+  const double t0 = trace_on() ? now_ms() : 0;
+  double t1 = 0, t2 = 0, t3 = 0;
   // line 3-4: V_mem / V_comp in ascending unit index: per-chunk counts (with max |S| and
   // the least nonzero |S| of each class, for the queue's key packing), then placement of
   // each unit and its S, all on the host cores
@@ -356,6 +370,7 @@ static void aorder_core(size_t n, SF S, AF active, uint32_t k, int order, uint32
     for (size_t i = 0; i < nmem; ++i) smem[i] = S(vmem[i]);
     for (size_t i = 0; i < ncomp; ++i) scomp[i] = S(vcomp[i]);
   }
+  if (trace_on()) t1 = now_ms();
   const size_t nact = nmem + ncomp;
   const size_t b = (nact + k - 1) / k;
   std::vector<int64_t> mem_sup(b, 0);        // line 1
@@ -391,6 +406,7 @@ static void aorder_core(size_t n, SF S, AF active, uint32_t k, int order, uint32
       q.replace_top(npk, live);                  // line 9
     }
     q.for_each([&](uint64_t pk) { mem_sup[pk & imask] = (int64_t)(pk >> ib) - off; });
+    if (trace_on()) t2 = now_ms();
     keys.clear();
     for (size_t i = 0; i < b; ++i)
       if (fill[i] < k) keys.push_back(pack(i, mem_sup[i], true));
@@ -432,6 +448,7 @@ static void aorder_core(size_t n, SF S, AF active, uint32_t k, int order, uint32
       q.update((size_t)bk, mem_sup[bk], alive[bk]);  // line 15
     }
   }
+  if (trace_on()) t3 = now_ms();
   // line 16-20: buckets in index order, members in insertion order (bucket start + rank);
   // inactive units last in unit order (Q16)
   bucket_off.assign(b + 1, 0);
@@ -445,6 +462,9 @@ static void aorder_core(size_t n, SF S, AF active, uint32_t k, int order, uint32
     uint32_t idx = inactive0 + (uint32_t)ci[t];
     for (size_t v = lo; v < hi; ++v) perm[v] = active(v) ? bucket_off[bucket_of[v]] + rank_of[v] : idx++;
   });
+  if (trace_on())
+    fprintf(stderr, "aorder n=%zu mem=%zu comp=%zu b=%zu: classify %.1f ms, phase1 %.1f, phase2 %.1f, relabel %.1f\n",
+            n, nmem, ncomp, b, t1 - t0, t2 - t1, t3 - t2, now_ms() - t3);
 }
 
 

@@ -134,11 +134,17 @@ __global__ void owners_total_kernel(const uint32_t *__restrict__ e1c, uint32_t n
   for (uint64_t x = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; x < n; x += (uint64_t)gridDim.x * blockDim.x)
     c[x] += e1c[x];
 }
+// E2 write cursor of x: its owner-list start plus its E1 owners
+__global__ void owners_cursor_kernel(const uint64_t *__restrict__ ooff, const uint32_t *__restrict__ e1c,
+                                     uint32_t n, unsigned long long *__restrict__ cur) {
+  for (uint64_t x = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; x < n; x += (uint64_t)gridDim.x * blockDim.x)
+    cur[x] = ooff[x] + e1c[x];
+}
 // owners of x: its E1 out-neighbours (N+(x) order) then its E2 in-neighbours (any order)
 __global__ void owners_scatter_kernel(const uint64_t *__restrict__ offs, const uint32_t *__restrict__ col,
                                       const uint32_t *__restrict__ od, uint32_t ub, uint32_t ue,
-                                      const uint64_t *__restrict__ ooff, const uint32_t *__restrict__ e1c,
-                                      uint32_t *__restrict__ e2p, uint32_t *__restrict__ own) {
+                                      const uint64_t *__restrict__ ooff, unsigned long long *__restrict__ e2cur,
+                                      uint32_t *__restrict__ own) {
   const uint64_t nw = (uint64_t)gridDim.x * (blockDim.x / 32);
   for (uint64_t u = ub + (uint64_t)blockIdx.x * (blockDim.x / 32) + warp_id(); u < ue; u += nw) {
     const uint64_t a = offs[u];
@@ -156,7 +162,7 @@ __global__ void owners_scatter_kernel(const uint64_t *__restrict__ offs, const u
       const unsigned m1 = __ballot_sync(0xffffffffu, e1);
       if (e1) own[p1 + __popc(m1 & ((1u << lane_id()) - 1u))] = v;
       p1 += __popc(m1);
-      if (j < du && dv > du) own[ooff[v] + e1c[v] + atomicAdd(&e2p[v], 1u)] = (uint32_t)u;
+      if (j < du && dv > du) own[atomicAdd(&e2cur[v], 1ull)] = (uint32_t)u;
     }
   }
 }
@@ -337,8 +343,12 @@ __global__ void edge_map_kernel(const uint64_t *__restrict__ offs, const uint32_
 
 // --------------------------------------------------------------- work model / analysis
 // w(u) = d~(u) + Σ_{v ∈ N+(u)} d~(v); sectors: 32-B sectors the Hu pattern touches with no reuse.
+// w[u] = d~(u) + Σ_{v ∈ N+(u)} d~(v) (the partition work model); sectors: the count's
+// algorithmic DRAM sectors with no reuse: per source with d~ >= 2 its
+// staged list + 1, per edge the streamed list + its offs pair — N+(v) (Hu's pattern), or
+// with `shorter` the shorter of N+(u), N+(v) (the shorter-list schedule of count_graph).
 __global__ void work_kernel(const uint64_t *__restrict__ offs, const uint32_t *__restrict__ col, uint32_t n,
-                            uint64_t *__restrict__ w, unsigned long long *sectors) {
+                            uint64_t *__restrict__ w, unsigned long long *sectors, int shorter) {
   uint64_t sec = 0;
   unsigned warps = gridDim.x * (blockDim.x / 32);
   for (uint64_t u = (uint64_t)blockIdx.x * (blockDim.x / 32) + warp_id(); u < n; u += warps) {
@@ -348,9 +358,11 @@ __global__ void work_kernel(const uint64_t *__restrict__ offs, const uint32_t *_
       uint32_t v = col[p];
       uint64_t vb = offs[v], ve = offs[v + 1];
       s += ve - vb;
-      // N+(v) list span + the offs pair
-      if (ve > vb) sc += ((ve * 4 - 1) >> 5) - ((vb * 4) >> 5) + 1;
-      sc += (((uint64_t)v * 8 + 15) >> 5) - (((uint64_t)v * 8) >> 5) + 1;
+      const bool own_u = shorter && ve - vb > e - a;  // E2: N+(u) is the streamed list
+      const uint64_t sb = own_u ? a : vb, se = own_u ? e : ve, sx = own_u ? u : v;
+      // streamed list span + its offs pair
+      if (se > sb) sc += ((se * 4 - 1) >> 5) - ((sb * 4) >> 5) + 1;
+      sc += ((sx * 8 + 15) >> 5) - ((sx * 8) >> 5) + 1;
     }
     s = warp_sum(s);
     sc = warp_sum(sc);
@@ -623,8 +635,9 @@ uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *
       // shorter-list owners (count modes, option "shorter"): per edge the shorter list is
       // streamed and searched in the longer one, which is staged once for all its owners
       Owners ow{nullptr, nullptr, 0, 0};
-      DevBuf<uint32_t> od_new, e1c, e2c, e2p, own;
+      DevBuf<uint32_t> od_new, e1c, e2c, own;
       DevBuf<uint64_t> ooff;
+      DevBuf<unsigned long long> e2cur;
       uint32_t iub = ub, iue = ue;  // sources of the item list
       // max d~ (label-free; from ensure_od when it ran, else from the CSR): with every list
       // short (max d~ < 64, e.g. ER) the two lists of an edge are alike and the owner pass
@@ -645,12 +658,12 @@ uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *
         }
         e1c.alloc(n, s);
         e2c.alloc(n, s);
-        e2p.alloc(n, s);
+        e2cur.alloc(n, s);
         ooff.alloc((uint64_t)n + 1, s);
         own.alloc(g.m ? g.m : 1, s);
+        ProfScope prof_owners("owners", s, 0.0);
         TC_CUDA(cudaMemsetAsync(e1c.get(), 0, e1c.bytes(), s));
         TC_CUDA(cudaMemsetAsync(e2c.get(), 0, e2c.bytes(), s));
-        TC_CUDA(cudaMemsetAsync(e2p.get(), 0, e2p.bytes(), s));
         const unsigned wgrid = grid_for((uint64_t)(ue - ub) * 32, 256, 8);
         owners_count_kernel<<<wgrid, 256, 0, s>>>(g.offs.get(), g.col.get(), od_new.get(), ub, ue, e1c.get(),
                                                   e2c.get());
@@ -658,10 +671,12 @@ uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *
         owners_total_kernel<<<grid_for(n, 256), 256, 0, s>>>(e1c.get(), n, e2c.get());
         TC_LAUNCH_CHECK();
         scan_u32_to_u64(e2c.get(), ooff.get(), n, s);
-        owners_scatter_kernel<<<wgrid, 256, 0, s>>>(g.offs.get(), g.col.get(), od_new.get(), ub, ue, ooff.get(),
-                                                    e1c.get(), e2p.get(), own.get());
+        owners_cursor_kernel<<<grid_for(n, 256), 256, 0, s>>>(ooff.get(), e1c.get(), n, e2cur.get());
         TC_LAUNCH_CHECK();
-        nlaunch += 5;
+        owners_scatter_kernel<<<wgrid, 256, 0, s>>>(g.offs.get(), g.col.get(), od_new.get(), ub, ue, ooff.get(),
+                                                    e2cur.get(), own.get());
+        TC_LAUNCH_CHECK();
+        nlaunch += 6;
         ow = Owners{ooff.get(), own.get(), (uint32_t)g_opt_owner_span, (uint32_t)g_opt_owner_lspan};
         iub = 0;  // an E2 edge u -> v is counted at v, any label
         iue = n;
@@ -844,7 +859,7 @@ void partition_graph(Graph &g, uint32_t world, uint32_t *bounds) {
   pre.alloc((uint64_t)n + 1, s);
   db.alloc(world + 1, s);
   if (n) {
-    work_kernel<<<grid_for((uint64_t)n * 32, 256), 256, 0, s>>>(g.offs.get(), g.col.get(), n, w.get(), nullptr);
+    work_kernel<<<grid_for((uint64_t)n * 32, 256), 256, 0, s>>>(g.offs.get(), g.col.get(), n, w.get(), nullptr, 0);
     TC_LAUNCH_CHECK();
   }
   scan_u64(w.get(), pre.get(), n, s);
@@ -864,7 +879,15 @@ void analyze_graph(Graph &g) {
   sec.alloc(1, s);
   TC_CUDA(cudaMemsetAsync(sec.get(), 0, 8, s));
   if (n) {
-    work_kernel<<<grid_for((uint64_t)n * 32, 256), 256, 0, s>>>(g.offs.get(), g.col.get(), n, w.get(), sec.get());
+    // the schedule count_graph runs for a plain count: shorter-list when max d~ >= 64
+    DevBuf<uint32_t> od_new;
+    od_new.alloc(n, s);
+    od_from_offs_kernel<<<grid_for(n, 256), 256, 0, s>>>(g.offs.get(), n, od_new.get());
+    TC_LAUNCH_CHECK();
+    const int shorter = g_opt_shorter && g_opt_intersect == 0 && device_max_u32(od_new.get(), n, s) >= 64;
+    g.alg_model_shorter = shorter;
+    work_kernel<<<grid_for((uint64_t)n * 32, 256), 256, 0, s>>>(g.offs.get(), g.col.get(), n, w.get(), sec.get(),
+                                                                shorter);
     TC_LAUNCH_CHECK();
   }
   scan_u64(w.get(), pre.get(), n, s);

@@ -21,7 +21,10 @@ constexpr uint32_t PIECE = 4096;      // large kernel: N+(u) piece in shared mem
 constexpr uint32_t LG_SUB = 8;        // large kernel: v's per dynamically fetched sub-chunk
 // bracket tables get 2^TS_* buckets per list element (finer buckets: fewer search steps)
 constexpr int TS_W = 2;               // warp items
-constexpr int TS_L = 1;               // CTA items (pieces)
+#ifndef TC_TS_L
+#define TC_TS_L 1
+#endif
+constexpr int TS_L = TC_TS_L;         // CTA items (pieces)
 constexpr uint32_t LG_SMEM_WORDS = (PIECE + 72) + ((PIECE << TS_L) + 64) / 2;  // piece (+pad) + u16 table
 constexpr uint32_t CHUNK = 8;         // worklist entries per atomic fetch
 
@@ -272,19 +275,62 @@ __device__ __forceinline__ void fast_block(const uint32_t *__restrict__ p, const
   }
 }
 
+// N consecutive 32-wedge steps spanning several owner lists (count modes): the owner of
+// wedge j is found without a per-lane walk — per step two warp reductions give the owners
+// starting at or before the step's first wedge (REDUX.ADD) and a bitmask of the owners
+// starting inside the step (REDUX.OR); a lane's owner is their sum up to its own offset.
+// st_lane: start (wedge index) of the owner list held by this lane, ~0 if none.  The tail is
+// clamped to the last wedge and its hits masked, as in wedge_block.
+template <int N, int MODE, class Search>
+__device__ __forceinline__ void wedge_block_rx(uint32_t base, uint32_t last, const uint32_t *__restrict__ col,
+                                               const Search &search, const WarpScratch &ws, uint32_t st_lane,
+                                               uint32_t &cnt) {
+  const uint32_t lane = lane_id();
+  uint32_t w[N];
+#pragma unroll
+  for (int k = 0; k < N; ++k) {
+    const uint32_t B = base + 32 * k;  // <= last for every step of a block
+    const uint32_t m = __reduce_or_sync(0xffffffffu, (st_lane - B - 1u) < 31u ? (1u << (st_lane - B)) : 0u);
+    const uint32_t c = __reduce_add_sync(0xffffffffu, st_lane <= B ? 1u : 0u);
+    const uint32_t off = min(lane, last - B);
+    const uint32_t o = c - 1u + __popc(m & ((2u << off) - 1u));
+    const uint32_t sto = o ? ws.pre[o - 1] : 0u;
+    w[k] = ldg_u32(col + ws.vb[o] + (B + off - sto));
+  }
+#pragma unroll
+  for (int k = 0; k < N; ++k) {
+    uint32_t pos;
+    const bool hit = search(w[k], pos) && base + 32 * k + lane <= last;
+    cnt += hit ? 1u : 0u;
+    if (MODE == 3) {  // §5.3 balance-point experiment, as in wedge_block
+      uint32_t acc = 0;
+      const uint32_t wi = ((base + lane) >> 5) + k;
+      const int ne = (int)((((uint64_t)wi + 1) * (uint32_t)g_extra) >> 3) - (int)(((uint64_t)wi * (uint32_t)g_extra) >> 3);
+      for (int e = 0; e < ne; ++e) {
+        uint32_t p2;
+        acc += search(w[k] ^ (uint32_t)(e + 1), p2) ? 1u : 0u;
+      }
+      cnt += acc & g_sink_mask;
+    }
+  }
+}
+
 // All wedges of one chunk in blocks of NB (8 for CTA items), 4, 2 and 1 steps of 32.  The
 // owner of each block's first wedge is tracked warp-uniformly; a block that lies entirely
 // in that owner's list (long N+(v): most wedges of a skewed graph) takes fast_block, the
 // others walk per lane from there (wedge_block).
 template <int MODE, class Search, int NB = 4>
 __device__ __forceinline__ uint32_t wedge_loop(const uint32_t *__restrict__ col, const Search &search, uint32_t sbase,
-                                               uint32_t cbase, uint32_t lo, uint32_t hi, uint32_t total,
+                                               uint32_t cbase, uint32_t st_lane, uint32_t total,
                                                WarpScratch &ws, unsigned long long *tv, uint64_t ebase) {
   constexpr bool FAST = MODE == 0 || MODE == 3 || MODE == 4;
   uint32_t cnt = 0;
   uint32_t uo = 0, uo_end = ws.pre[0];
   const uint32_t *uob = col + ws.vb[0];  // element j of the uniform owner's list is uob[j]
   const uint32_t last = total - 1, steps = (total + 31) >> 5, lane = lane_id();
+  // owner lists averaging < 8 wedges: a per-lane walk would cross several owners per step,
+  // so the owners are located by warp reductions instead (wedge_block_rx)
+  const bool short_lists = FAST && total < 8u * (uint32_t)__popc(__ballot_sync(0xffffffffu, st_lane != 0xffffffffu));
   auto block = [&](auto nconst, uint32_t st) {
     constexpr int N = decltype(nconst)::value;
     const uint32_t base = 32 * st;
@@ -296,6 +342,8 @@ __device__ __forceinline__ uint32_t wedge_loop(const uint32_t *__restrict__ col,
     }
     if (FAST && uo_end >= base + 32 * N) {
       fast_block<N, MODE>(uob + base + lane, search, base + lane, cnt);
+    } else if (FAST && short_lists) {
+      wedge_block_rx<N, MODE>(base, last, col, search, ws, st_lane, cnt);
     } else {
       uint32_t o = uo, o_end = uo_end;
       const uint32_t *ob = uob;
@@ -311,8 +359,6 @@ __device__ __forceinline__ uint32_t wedge_loop(const uint32_t *__restrict__ col,
     st += 2;
   }
   if (st < steps) block(std::integral_constant<int, 1>(), st);
-  (void)lo;
-  (void)hi;
   return cnt;
 }
 
@@ -377,6 +423,7 @@ __device__ __forceinline__ uint32_t warp_chunk(const uint64_t *__restrict__ offs
   const uint32_t inc = warp_inclusive_scan(dv);
   const uint32_t total = __shfl_sync(0xffffffffu, inc, 31);
   const unsigned nz = __ballot_sync(0xffffffffu, dv != 0);
+  const uint32_t st_lane = dv ? inc - dv : 0xffffffffu;  // wedge index where this lane's list starts
   if (dv) {
     const unsigned pos = __popc(nz & ((1u << lane) - 1u));
     ws.vb[pos] = vb;
@@ -401,7 +448,7 @@ __device__ __forceinline__ uint32_t warp_chunk(const uint64_t *__restrict__ offs
     if (MODE == 4) {  // every staged list has <= 32 entries (host-checked): 1..5 steps only
       switch (S) {
 #define TC_SHORT(k) \
-  case k: cnt = wedge_loop<MODE, Pow2Search<k>, NB>(col, Pow2Search<k>{smem_addr(sbase), sbase}, sbase, cbase, lo, hi, total, ws, tv, ebase); break;
+  case k: cnt = wedge_loop<MODE, Pow2Search<k>, NB>(col, Pow2Search<k>{smem_addr(sbase), sbase}, sbase, cbase, st_lane, total, ws, tv, ebase); break;
         TC_SHORT(1) TC_SHORT(2) TC_SHORT(3) TC_SHORT(4) TC_SHORT(5)
 #undef TC_SHORT
       }
@@ -411,12 +458,12 @@ __device__ __forceinline__ uint32_t warp_chunk(const uint64_t *__restrict__ offs
   case k:                                                                                                    \
     if (abs_t)                                                                                               \
       cnt = wedge_loop<MODE, TabSearch<k, true>, NB>(                                                        \
-          col, TabSearch<k, true>{smem_addr(sbase), smem_addr(tbase), 0u, sh, 0u, sbase}, sbase, cbase, lo, hi, \
+          col, TabSearch<k, true>{smem_addr(sbase), smem_addr(tbase), 0u, sh, 0u, sbase}, sbase, cbase, st_lane, \
           total, ws, tv, ebase);                                                                             \
     else                                                                                                     \
       cnt = wedge_loop<MODE, TabSearch<k, false>, NB>(                                                       \
           col, TabSearch<k, false>{smem_addr(sbase), smem_addr(tbase), tlo, sh, ((thi - tlo) >> sh) + 1, sbase}, \
-          sbase, cbase, lo, hi, total, ws, tv, ebase);                                                       \
+          sbase, cbase, st_lane, total, ws, tv, ebase);                                                       \
     break;
         TC_TAB(0) TC_TAB(1) TC_TAB(2) TC_TAB(3) TC_TAB(4) TC_TAB(5) TC_TAB(6)
 #undef TC_TAB
@@ -424,12 +471,12 @@ __device__ __forceinline__ uint32_t warp_chunk(const uint64_t *__restrict__ offs
     } else {
       switch (S) {
 #define TC_CASE(k) \
-  case k: cnt = wedge_loop<MODE, Pow2Search<k>, NB>(col, Pow2Search<k>{smem_addr(sbase), sbase}, sbase, cbase, lo, hi, total, ws, tv, ebase); break;
+  case k: cnt = wedge_loop<MODE, Pow2Search<k>, NB>(col, Pow2Search<k>{smem_addr(sbase), sbase}, sbase, cbase, st_lane, total, ws, tv, ebase); break;
         TC_CASE(1) TC_CASE(2) TC_CASE(3) TC_CASE(4) TC_CASE(5) TC_CASE(6) TC_CASE(7)
         TC_CASE(8) TC_CASE(9) TC_CASE(10) TC_CASE(11) TC_CASE(12) TC_CASE(13) TC_CASE(14)
 #undef TC_CASE
         default:
-          cnt = wedge_loop<MODE, GlobalSearch, NB>(col, GlobalSearch{list, L, sbase}, sbase, 0xffffffffu, lo, hi, total, ws, tv, ebase);
+          cnt = wedge_loop<MODE, GlobalSearch, NB>(col, GlobalSearch{list, L, sbase}, sbase, 0xffffffffu, st_lane, total, ws, tv, ebase);
       }
     }
   }
@@ -437,6 +484,9 @@ __device__ __forceinline__ uint32_t warp_chunk(const uint64_t *__restrict__ offs
   if (PV && lane < (unsigned)__popc(nz) && ws.vcnt[lane]) atomicAdd(&tv[ws.v[lane]], (unsigned long long)ws.vcnt[lane]);
   if (PE && lane < (unsigned)__popc(nz) && ws.vcnt[lane])
     atomicAdd(&tv[ua + ws.v[lane]], (unsigned long long)ws.vcnt[lane]);
+  // the flush reads ws.v / ws.vcnt of other owners: order it before the next chunk's writes
+  // (compute-sanitizer racecheck WAR hazard across consecutive chunks of a CTA item)
+  if (PV || PE) __syncwarp();
   return cnt;
 }
 

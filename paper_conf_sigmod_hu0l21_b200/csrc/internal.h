@@ -75,6 +75,7 @@ struct Graph {
 
   // results / stats
   uint64_t triangles = 0, wedges = 0, alg_bytes = 0;
+  int alg_model_shorter = 0;  // alg_bytes modelled the shorter-list schedule (tc_analyze)
   double ms_build = 0, ms_direct = 0, ms_reorder = 0, ms_count = 0, ms_count_kernel = 0;
   uint64_t count_launches = 0;
 };

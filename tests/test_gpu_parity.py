@@ -278,12 +278,15 @@ def test_bench_under_torchrun_single_process():
     root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
     cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "1",
            "--master-addr", "127.0.0.1", "--master-port", "29533", os.path.join(root, "bench.py"),
-           "--gpus", "1", "--steps", "2", "--warmup", "1", "--config", "1", "--no-e2e", "--no-cpu-baseline"]
+           "--gpus", "1", "--steps", "2", "--warmup", "1", "--config", "1", "--reorder", "paper", "--no-e2e",
+           "--no-cpu-baseline"]
     env = dict(os.environ, WORLD_SIZE="1")
     out = subprocess.run(cmd, capture_output=True, text=True, timeout=600, env=env, cwd=root)
     assert out.returncode == 0, out.stderr[-2000:]
     line = json.loads(out.stdout.strip().splitlines()[-1])
     assert line["config"]["triangles"] > 0 and line["value"] > 0
+    # t = max over ranks of (count + allreduce); A-order broadcast from rank 0
+    assert "allreduce" in line["value_def"] and "ncclBroadcast" in line["config"]["parallelism"]
 
 
 # ---------------------------------------------------------------- per-edge support (f1)
@@ -453,3 +456,74 @@ def test_edge_aorder_schedule(d, r):
         g = tc.Graph(src, dst, N).direct(d).reorder(r).set_schedule("edge_aorder")
         assert g.count() == T, name
         g.free()
+
+
+# ---------------------------------------------------------------- shorter-list schedule, options
+@pytest.mark.parametrize("cap", [32, 256])
+@pytest.mark.parametrize("spans", [(32, 8), (128, 2048), (1 << 12, 1 << 16)])
+def test_shorter_list_schedule(cap, spans):
+    """Count with the shorter-list owner schedule (default for count-only calls) and with the
+    classic Hu pattern: every warp / CTA owner-item shape gives the oracle's T, whole and on
+    work-balanced slices (the owners of a slice are its sources' edges, counted at either end)."""
+    span, lspan = spans
+    tc.tc_set_option("small_cap", cap)
+    tc.tc_set_option("owner_span", span)
+    tc.tc_set_option("owner_lspan", lspan)
+    try:
+        for seed, (sc, ef, d, r) in enumerate(((13, 16, "degree", "none"), (12, 32, "paper", "paper"),
+                                               (12, 16, "id", "degree"))):
+            spec = graphgen.rmat_spec(sc, ef, 900 + seed)
+            src, dst = graphgen.generate_cpu(spec)
+            ref = oracle.run(src, dst, spec.n, d, r)
+            g = tc.Graph(src, dst, spec.n).direct(d).reorder(r)
+            for shorter in (1, 0):
+                tc.tc_set_option("shorter", shorter)
+                assert g.count() == ref["T"], (d, r, shorter)
+                b = g.partition(3).tolist()
+                assert sum(g.count_range(a, c) for a, c in zip(b, b[1:])) == ref["T"]
+            g.free()
+    finally:
+        tc.tc_set_option("shorter", 1)
+        tc.tc_set_option("small_cap", 256)
+        tc.tc_set_option("owner_span", 128)
+        tc.tc_set_option("owner_lspan", 2048)
+
+
+def test_extra_compute_instrumented_kernel_counts_unchanged():
+    """The §5.3 balance-point instrumentation (option extra_compute, MODE 3: p_c extra
+    searches per wedge, results discarded) leaves T and t(v) equal to the oracle's."""
+    spec = graphgen.rmat_spec(12, 16, 31)
+    src, dst = graphgen.generate_cpu(spec)
+    ref = oracle.run(src, dst, spec.n, "degree", "paper", per_vertex=True)
+    g = tc.Graph(src, dst, spec.n).direct("degree").reorder("paper")
+    try:
+        for q in (0, 1, 8, 24):
+            tc.tc_set_option("extra_compute", q)
+            assert g.count() == ref["T"], q
+            T, t = g.count(per_vertex=True)
+            assert T == ref["T"] and np.array_equal(t, ref["t"]), q
+    finally:
+        tc.tc_set_option("extra_compute", -1)
+        g.free()
+
+
+def test_reorder_dist_single_rank_equals_reorder():
+    """tc_reorder_dist (A-order on rank 0, pi / bucket_off / Eq.3 broadcast over NCCL) gives
+    the same graph as tc_reorder, and the count through tc_count_dist equals the oracle's."""
+    spec = graphgen.rmat_spec(13, 16, 41)
+    src, dst = graphgen.generate_cpu(spec)
+    ref = oracle.run(src, dst, spec.n, "degree", "paper")
+    uid = tc.tc_nccl_get_unique_id()
+    comm = tc.tc_nccl_comm_init(uid, 0, 1, 0)
+    try:
+        g = tc.Graph(src, dst, spec.n).direct("degree")
+        prm, keep = tc.make_aorder_params()
+        tc.tc_reorder_dist(g.handle, "paper", prm, comm, 0, 1)
+        offs, col, perm = g.export()
+        assert np.array_equal(perm, ref["perm"]) and np.array_equal(col, ref["col"])
+        assert np.array_equal(g.export_buckets(), ref["bucket_off"])
+        assert g.stats()["eq3"] == oracle.objective_eq3(ref["bucket_off"], ref["perm"], ref["od"])
+        assert tc.tc_count_dist(g.handle, comm, 0, 1) == ref["T"]
+        g.free()
+    finally:
+        tc.tc_nccl_comm_destroy(comm)

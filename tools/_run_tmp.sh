@@ -1,5 +1,7 @@
 set -u
 OUT=gpurun_out; mkdir -p $OUT
-TAG=r02d STEPS="tests bench launches full" bash tools/gpu_round.sh
-for c in 3 2 5; do timeout 900 python bench.py --config $c --no-e2e --no-cpu-baseline --steps 3 --warmup 2 > $OUT/r02d_bench_cfg$c.json 2>&1; python -c "
-import json; d=json.load(open('$OUT/r02d_bench_cfg$c.json')); print($c, d['value'], d['count_ms'], d['whole_path'], d['stages_ms'])"; done
+timeout 900 python -m pytest tests/test_gpu_parity.py -x -q -k "shorter or closed or random or config1 or multi_piece or schedules" > $OUT/r02h_pytest.log 2>&1; echo "rc=$?" >> $OUT/r02h_pytest.log
+tail -2 $OUT/r02h_pytest.log
+python tools/kprof.py --config 4 --rule degree:paper --reps 2 2>&1 | head -3
+python tools/kprof.py --config 3 --rule paper:none --reps 3 2>&1 | head -3
+python tools/kprof.py --config 5 --rule paper:paper --reps 1 2>&1 | head -3

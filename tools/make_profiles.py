@@ -41,7 +41,8 @@ def launches(path):
             continue
         v = float(d["Metric Value"].replace(",", ""))
         unit = d["Metric Unit"]
-        v *= {"nsecond": 1e-3, "usecond": 1.0, "msecond": 1e3, "second": 1e6}.get(unit, 1.0)
+        v *= {"nsecond": 1e-3, "ns": 1e-3, "usecond": 1.0, "us": 1.0, "msecond": 1e3, "ms": 1e3,
+              "second": 1e6, "s": 1e6}.get(unit, 1.0)
         a = agg.setdefault(kernel_short(d["Kernel Name"]), [0, 0.0])
         a[0] += 1
         a[1] += v
@@ -49,7 +50,11 @@ def launches(path):
 
 
 def full(path):
-    out = subprocess.run(["ncu", "-i", path, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
+    """Summary of one `ncu --page raw --csv` page (a .raw.csv file, or a .ncu-rep read with ncu)."""
+    if path.endswith(".ncu-rep"):
+        out = subprocess.run(["ncu", "-i", path, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
+    else:
+        out = open(path).read()
     rows = list(csv.reader(io.StringIO(out)))
     if len(rows) < 3:
         return None
@@ -75,11 +80,12 @@ def main():
     ap.add_argument("--cfg", type=int, default=2)
     ap.add_argument("--rules", default="degree:none")
     ap.add_argument("--src", default=os.path.join(ROOT, "gpurun_out"))
+    ap.add_argument("--tag", default="", help="file prefix of tools/gpu_round.sh outputs, e.g. r02d_")
     a = ap.parse_args()
     prof = os.path.join(ROOT, "profiles")
     os.makedirs(prof, exist_ok=True)
     lines = [f"# {a.round}: ncu summary, BASELINE configs[{a.cfg - 1}] ({a.rules})", ""]
-    lp = os.path.join(a.src, f"launches_cfg{a.cfg}.csv")
+    lp = os.path.join(a.src, f"{a.tag}launches_cfg{a.cfg}.csv")
     if os.path.exists(lp):
         agg = launches(lp)
         tot = sum(t for _, t in agg.values())
@@ -89,7 +95,8 @@ def main():
             lines.append(f"| {k} | {c} | {t:.1f} | {100 * t / tot:.1f}% |")
         lines.append("")
     traffic = {}
-    for p in sorted(glob.glob(os.path.join(a.src, f"full_cfg{a.cfg}_*.ncu-rep"))):
+    for p in sorted(glob.glob(os.path.join(a.src, f"{a.tag}full_cfg{a.cfg}_*.ncu-rep")) +
+                    glob.glob(os.path.join(a.src, f"{a.tag}full_cfg{a.cfg}_*.raw.csv"))):
         r = full(p)
         if not r:
             continue
@@ -100,10 +107,11 @@ def main():
         lines.append("- top stalls (warps per issue): " + ", ".join(f"{n} {v:.2f}" for v, n in r["stalls"]))
         lines.append(f"- DRAM traffic per launch: {r['traffic_bytes'] / 1e6:.1f} MB")
         lines.append("")
-        name = {"rs_pass_kernel": "radix_pass", "count_small_kernel": "count", "count_range_kernel": "count",
-                "count_large_kernel": "count_large", "unique_kernel": "unique",
+        name = {"rs_pass_kernel": "radix_pass", "unique_kernel": "unique",
                 "rs_hist_kernel": "radix_hist"}.get(r["kernel"], r["kernel"])
         traffic[name] = r["traffic_bytes"]
+        if r["kernel"].startswith("count_"):  # the count kernels share one bytes model (bench "count")
+            traffic["count"] = traffic.get("count", 0.0) + r["traffic_bytes"]
     with open(os.path.join(prof, f"{a.round}_ncu_cfg{a.cfg}.md"), "w") as f:
         f.write("\n".join(lines) + "\n")
     tj = os.path.join(prof, "traffic.json")
