@@ -200,6 +200,9 @@ tc_status tc_set_option(const char *key, int64_t value) {
     else if (k == "owner_span") {
       TC_REQUIRE(value >= 32 && value <= (1 << 20) && value % 32 == 0, ST_INVALID, "owner_span: multiple of 32");
       g_opt_owner_span = (int)value;
+    } else if (k == "vtiles") {
+      TC_REQUIRE(value >= 1 && value <= 1024, ST_INVALID, "vtiles: 1 .. 1024");
+      g_opt_vtiles = (int)value;
     } else if (k == "owner_lspan") {
       TC_REQUIRE(value >= 8 && value <= (1 << 24), ST_INVALID, "owner_lspan: 8 .. 2^24");
       g_opt_owner_lspan = (int)value;

@@ -41,6 +41,7 @@ int g_opt_l2_persist = 0;    // L2 access-policy window over [offs | col] during
 int g_opt_shorter = 1;       // count modes: per edge the shorter list is streamed (owner lists)
 int g_opt_owner_span = 128;  // owners per warp item (shorter-list schedule)
 int g_opt_owner_lspan = 2048;  // owners per CTA item
+int g_opt_vtiles = 1;        // classic count: streamed lists in this many L2 label tiles (1 = off)
 
 using namespace cnt;
 namespace {
@@ -634,7 +635,7 @@ uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *
     } else {
       // shorter-list owners (count modes, option "shorter"): per edge the shorter list is
       // streamed and searched in the longer one, which is staged once for all its owners
-      Owners ow{nullptr, nullptr, 0, 0};
+      Owners ow{nullptr, nullptr, 0, 0, 0, 0xffffffffu};
       DevBuf<uint32_t> od_new, e1c, e2c, own;
       DevBuf<uint64_t> ooff;
       DevBuf<unsigned long long> e2cur;
@@ -677,7 +678,7 @@ uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *
                                                     e2cur.get(), own.get());
         TC_LAUNCH_CHECK();
         nlaunch += 6;
-        ow = Owners{ooff.get(), own.get(), (uint32_t)g_opt_owner_span, (uint32_t)g_opt_owner_lspan};
+        ow = Owners{ooff.get(), own.get(), (uint32_t)g_opt_owner_span, (uint32_t)g_opt_owner_lspan, 0, 0xffffffffu};
         iub = 0;  // an E2 edge u -> v is counted at v, any label
         iue = n;
       }
@@ -747,9 +748,20 @@ uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *
           uint64_t want = (nsmall + CT_WARPS - 1) / CT_WARPS;
           unsigned grid = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(want, (uint64_t)num_sms() * occ));
           ProfScope prof("count_small", s, 0.0);
-          launch(small_fn, grid, CT_THREADS, smem, s, (const uint64_t *)g.offs.get(), (const uint32_t *)g.col.get(),
-                 (const uint64_t *)(items.get() + nlarge), nsmall, nheavy, hist.get() + 65, cap_small,
-                 (unsigned long long *)dT.get(), tv, vbits, ow);
+          // option "vtiles" (classic schedule, count modes, no CTA items): the streamed lists
+          // N+(v) in label tiles counted one pass each, so a tile's lists stay in L2
+          const uint32_t tiles = (!ow.own && (mode == 0) && !nlarge && g_opt_vtiles > 1) ? (uint32_t)g_opt_vtiles : 1u;
+          for (uint32_t t = 0; t < tiles; ++t) {
+            Owners owt = ow;
+            if (tiles > 1) {
+              owt.vlo = (uint32_t)((uint64_t)g.n * t / tiles);
+              owt.vhi = (uint32_t)((uint64_t)g.n * (t + 1) / tiles);
+              if (t) TC_CUDA(cudaMemsetAsync(hist.get() + 65, 0, 2 * sizeof(unsigned long long), s));
+            }
+            launch(small_fn, grid, CT_THREADS, smem, s, (const uint64_t *)g.offs.get(), (const uint32_t *)g.col.get(),
+                   (const uint64_t *)(items.get() + nlarge), nsmall, nheavy, hist.get() + 65, cap_small,
+                   (unsigned long long *)dT.get(), tv, vbits, owt);
+          }
           ++nlaunch;
         }
         if (kernel_ms) TC_CUDA(cudaEventRecord(e1, s));

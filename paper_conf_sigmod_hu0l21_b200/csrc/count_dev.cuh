@@ -19,6 +19,13 @@ constexpr int LG_THREADS = 256;       // large kernel: 8 warps
 constexpr int LG_WARPS = LG_THREADS / 32;
 constexpr uint32_t PIECE = 4096;      // large kernel: N+(u) piece in shared memory (16 KB)
 constexpr uint32_t LG_SUB = 8;        // large kernel: v's per dynamically fetched sub-chunk
+#ifndef TC_LG_SUB_OWN
+#define TC_LG_SUB_OWN 32
+#endif
+constexpr uint32_t LG_SUB_OWN = TC_LG_SUB_OWN;  // ... of the shorter-list schedule (owners)
+#ifndef TC_LG_MINB_OWN
+#define TC_LG_MINB_OWN 5
+#endif
 // bracket tables get 2^TS_* buckets per list element (finer buckets: fewer search steps)
 constexpr int TS_W = 2;               // warp items
 #ifndef TC_TS_L
@@ -45,6 +52,9 @@ struct Owners {
   const uint64_t *off;  // off[x] .. off[x+1]: owners of x in own[]
   const uint32_t *own;
   uint32_t span, lspan;
+  // classic schedule, count modes: only v in [vlo, vhi) this pass (L2 tiles of the
+  // streamed lists, option "vtiles"); [0, 2^32) = every v
+  uint32_t vlo = 0, vhi = 0xffffffffu;
 };
 
 __device__ __forceinline__ uint32_t ldg_u32(const uint32_t *p) { return __ldg(p); }
@@ -275,46 +285,6 @@ __device__ __forceinline__ void fast_block(const uint32_t *__restrict__ p, const
   }
 }
 
-// N consecutive 32-wedge steps spanning several owner lists (count modes): the owner of
-// wedge j is found without a per-lane walk — per step two warp reductions give the owners
-// starting at or before the step's first wedge (REDUX.ADD) and a bitmask of the owners
-// starting inside the step (REDUX.OR); a lane's owner is their sum up to its own offset.
-// st_lane: start (wedge index) of the owner list held by this lane, ~0 if none.  The tail is
-// clamped to the last wedge and its hits masked, as in wedge_block.
-template <int N, int MODE, class Search>
-__device__ __forceinline__ void wedge_block_rx(uint32_t base, uint32_t last, const uint32_t *__restrict__ col,
-                                               const Search &search, const WarpScratch &ws, uint32_t st_lane,
-                                               uint32_t &cnt) {
-  const uint32_t lane = lane_id();
-  uint32_t w[N];
-#pragma unroll
-  for (int k = 0; k < N; ++k) {
-    const uint32_t B = base + 32 * k;  // <= last for every step of a block
-    const uint32_t m = __reduce_or_sync(0xffffffffu, (st_lane - B - 1u) < 31u ? (1u << (st_lane - B)) : 0u);
-    const uint32_t c = __reduce_add_sync(0xffffffffu, st_lane <= B ? 1u : 0u);
-    const uint32_t off = min(lane, last - B);
-    const uint32_t o = c - 1u + __popc(m & ((2u << off) - 1u));
-    const uint32_t sto = o ? ws.pre[o - 1] : 0u;
-    w[k] = ldg_u32(col + ws.vb[o] + (B + off - sto));
-  }
-#pragma unroll
-  for (int k = 0; k < N; ++k) {
-    uint32_t pos;
-    const bool hit = search(w[k], pos) && base + 32 * k + lane <= last;
-    cnt += hit ? 1u : 0u;
-    if (MODE == 3) {  // §5.3 balance-point experiment, as in wedge_block
-      uint32_t acc = 0;
-      const uint32_t wi = ((base + lane) >> 5) + k;
-      const int ne = (int)((((uint64_t)wi + 1) * (uint32_t)g_extra) >> 3) - (int)(((uint64_t)wi * (uint32_t)g_extra) >> 3);
-      for (int e = 0; e < ne; ++e) {
-        uint32_t p2;
-        acc += search(w[k] ^ (uint32_t)(e + 1), p2) ? 1u : 0u;
-      }
-      cnt += acc & g_sink_mask;
-    }
-  }
-}
-
 // All wedges of one chunk in blocks of NB (8 for CTA items), 4, 2 and 1 steps of 32.  The
 // owner of each block's first wedge is tracked warp-uniformly; a block that lies entirely
 // in that owner's list (long N+(v): most wedges of a skewed graph) takes fast_block, the
@@ -328,9 +298,7 @@ __device__ __forceinline__ uint32_t wedge_loop(const uint32_t *__restrict__ col,
   uint32_t uo = 0, uo_end = ws.pre[0];
   const uint32_t *uob = col + ws.vb[0];  // element j of the uniform owner's list is uob[j]
   const uint32_t last = total - 1, steps = (total + 31) >> 5, lane = lane_id();
-  // owner lists averaging < 8 wedges: a per-lane walk would cross several owners per step,
-  // so the owners are located by warp reductions instead (wedge_block_rx)
-  const bool short_lists = FAST && total < 8u * (uint32_t)__popc(__ballot_sync(0xffffffffu, st_lane != 0xffffffffu));
+  (void)st_lane;  // (a warp-reduction owner lookup for short lists was measured slower)
   auto block = [&](auto nconst, uint32_t st) {
     constexpr int N = decltype(nconst)::value;
     const uint32_t base = 32 * st;
@@ -342,8 +310,6 @@ __device__ __forceinline__ uint32_t wedge_loop(const uint32_t *__restrict__ col,
     }
     if (FAST && uo_end >= base + 32 * N) {
       fast_block<N, MODE>(uob + base + lane, search, base + lane, cnt);
-    } else if (FAST && short_lists) {
-      wedge_block_rx<N, MODE>(base, last, col, search, ws, st_lane, cnt);
     } else {
       uint32_t o = uo, o_end = uo_end;
       const uint32_t *ob = uob;
@@ -569,8 +535,9 @@ __device__ __forceinline__ uint64_t warp_item(const uint64_t *__restrict__ offs,
     list = col + a;
   }
   const uint32_t lo = list[0], hi = list[L - 1];
-  const bool valid = c0 + lane < L;
+  bool valid = c0 + lane < L;
   const uint32_t v = valid ? list[c0 + lane] : 0u;
+  if (MODE == 0 || MODE == 4) valid = valid && v - ow.vlo < ow.vhi - ow.vlo;  // v-tile pass
   uint32_t cnt = warp_chunk<MODE>(offs, col, v, valid, list, sbase, padded ? sbase + cap + 64 : 0xffffffffu, cbase, L,
                                   padded, lo, hi, ws, tv, c0 + lane, a, a, vbits);
   __syncwarp();  // slice reads done before the next item restages it
@@ -696,7 +663,7 @@ __device__ __forceinline__ void mbar_wait(uint64_t *bar, unsigned phase) {
 // CTA items (u, c0) of heavy sources: v's N+(u)[c0 .. c0+LV) over 16 warps; N+(u) staged
 // piece by piece with a TMA bulk copy (cp.async.bulk + mbarrier complete_tx).
 template <int MODE, bool OWN = false>
-__global__ __launch_bounds__(LG_THREADS, 5) void count_large_kernel(const uint64_t *__restrict__ offs,
+__global__ __launch_bounds__(LG_THREADS, OWN ? TC_LG_MINB_OWN : 5) void count_large_kernel(const uint64_t *__restrict__ offs,
                                                                  const uint32_t *__restrict__ col,
                                                                  const uint64_t *__restrict__ items, uint64_t nitems,
                                                                  unsigned long long *ctr, unsigned long long *T,
@@ -791,9 +758,10 @@ __global__ __launch_bounds__(LG_THREADS, 5) void count_large_kernel(const uint64
       while (true) {
         uint32_t sc = 0;
         if (lane_id() == 0) sc = atomicAdd(&s_next, 1u);
-        const uint32_t c0 = cbeg + __shfl_sync(0xffffffffu, sc, 0) * LG_SUB;
+        constexpr uint32_t SUB = OWN ? LG_SUB_OWN : LG_SUB;
+        const uint32_t c0 = cbeg + __shfl_sync(0xffffffffu, sc, 0) * SUB;
         if (c0 >= cend) break;
-        const bool valid = lane_id() < LG_SUB && c0 + lane_id() < cend;
+        const bool valid = lane_id() < SUB && c0 + lane_id() < cend;
         const uint32_t v = valid ? ldg_u32(olist + c0 + lane_id()) : 0u;
         cnt += warp_chunk<MODE, MODE == 0 ? 8 : 4>(offs, col, v, valid, list, shift, S2 >= 0 ? tbase_lg : 0xffffffffu, 0xffffffffu, plen,
                                 true, lo, hi, ws, tv, c0 + lane_id(), a, a + p0, vbits, S2 >= 0 ? S2 : -2, sh,

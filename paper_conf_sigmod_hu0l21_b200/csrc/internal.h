@@ -135,5 +135,6 @@ extern int g_opt_split;  // orientation split CSR build (original labels)
 extern int g_opt_shorter;      // shorter-list owner schedule for count modes
 extern int g_opt_owner_span;   // owners per warp item
 extern int g_opt_owner_lspan;  // owners per CTA item
+extern int g_opt_vtiles;       // classic count: label tiles of the streamed lists (1 = off)
 
 }  // namespace tc
