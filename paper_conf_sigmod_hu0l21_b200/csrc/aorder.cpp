@@ -122,6 +122,7 @@ struct PackedTournament4 {
 // an exact binary min-heap (small, cache-resident), higher bins are plain vectors.
 struct MonoQueue {
   int shift = 0;
+  int lo_bits = 0;  // low key bits below the value (the bucket index)
   uint64_t bin0 = 0;
   std::vector<std::vector<uint64_t>> bins;
   // the current (lowest non-empty) bin, sorted once when it becomes current: it is then
@@ -165,7 +166,10 @@ struct MonoQueue {
     }
     heap[i] = x;
   }
-  // LSD radix sort of the current bin on its low `shift` bits (the high bits are the bin)
+  // Sort of the current bin: LSD radix on the value bits below the bin boundary only
+  // ([lo_bits, shift): the bin fixes the bits above, the low lo_bits are the bucket index),
+  // stable; then every run of equal values is put in index order (rare, except for the
+  // initial all-zero bin, which is already in index order)
   void sort_run() {
     const size_t n = run.size();
     if (n < 64) {
@@ -174,17 +178,25 @@ struct MonoQueue {
     }
     tmp.resize(n);
     uint32_t cnt[256];
-    for (int b = 0; b < shift; b += 8) {
+    for (int b = lo_bits; b < shift; b += 8) {
+      const int w = std::min(8, shift - b);
+      const uint64_t mask = (1ull << w) - 1;
       std::fill(cnt, cnt + 256, 0u);
-      for (size_t i = 0; i < n; ++i) ++cnt[(run[i] >> b) & 255];
+      for (size_t i = 0; i < n; ++i) ++cnt[(run[i] >> b) & mask];
       uint32_t acc = 0;
-      for (int d = 0; d < 256; ++d) {
+      for (uint64_t d = 0; d <= mask; ++d) {
         const uint32_t c = cnt[d];
         cnt[d] = acc;
         acc += c;
       }
-      for (size_t i = 0; i < n; ++i) tmp[cnt[(run[i] >> b) & 255]++] = run[i];
+      for (size_t i = 0; i < n; ++i) tmp[cnt[(run[i] >> b) & mask]++] = run[i];
       run.swap(tmp);
+    }
+    for (size_t i = 0; i < n;) {
+      size_t j = i + 1;
+      while (j < n && (run[j] >> lo_bits) == (run[i] >> lo_bits)) ++j;
+      if (j - i > 1 && !std::is_sorted(run.begin() + i, run.begin() + j)) std::sort(run.begin() + i, run.begin() + j);
+      i = j;
     }
   }
   void refill() {
@@ -198,7 +210,8 @@ struct MonoQueue {
   }
   // keys: packed keys of the alive buckets; max_pk: upper bound of any key ever inserted;
   // step: smallest key increment (packed units).  Bins ~step/8 wide (<= 2^16 bins).
-  void build(const std::vector<uint64_t> &keys, uint64_t max_pk, uint64_t step) {
+  void build(const std::vector<uint64_t> &keys, uint64_t max_pk, uint64_t step, int low_bits) {
+    lo_bits = low_bits;
     uint64_t mn = UINT64_MAX;
     for (uint64_t k : keys) mn = std::min(mn, k);
     if (keys.empty()) mn = 0;
@@ -393,7 +406,7 @@ static void aorder_core(size_t n, SF S, AF active, uint32_t k, int order, uint32
     std::vector<uint64_t> keys;
     keys.reserve(b);
     for (size_t i = 0; i < b; ++i) keys.push_back(pack(i, 0, false));
-    q.build(keys, max_pk, smin1 == INT64_MAX ? 0 : (uint64_t)smin1 << ib);  // line 2: min queue
+    q.build(keys, max_pk, smin1 == INT64_MAX ? 0 : (uint64_t)smin1 << ib, ib);  // line 2: min queue
     for (size_t i = 0; i < nmem; ++i) {          // line 5
       const uint64_t pk = q.top();
       const size_t bk = (size_t)(pk & imask);    // line 6
@@ -410,7 +423,7 @@ static void aorder_core(size_t n, SF S, AF active, uint32_t k, int order, uint32
     keys.clear();
     for (size_t i = 0; i < b; ++i)
       if (fill[i] < k) keys.push_back(pack(i, mem_sup[i], true));
-    q.build(keys, max_pk, smin2 == INT64_MAX ? 0 : (uint64_t)smin2 << ib);  // line 10: max queue
+    q.build(keys, max_pk, smin2 == INT64_MAX ? 0 : (uint64_t)smin2 << ib, ib);  // line 10: max queue
     for (size_t i = 0; i < ncomp; ++i) {         // line 11
       const uint64_t pk = q.top();
       const size_t bk = (size_t)(pk & imask);    // line 12
