@@ -167,7 +167,9 @@ tc_status tc_count_range(tc_graph *g, uint32_t u_begin, uint32_t u_end, uint64_t
                          uint64_t *per_vertex);
 
 /* Work-balanced contiguous ranges for `world` GPUs: bounds[0..world], bounds[0]=0,
- * bounds[world]=n (host memory).  Work model w(u) = d~(u) + sum_{v in N+(u)} d~(v). */
+ * bounds[world]=n (host memory).  Work model = the elements the count streams for the
+ * source's edges: w(u) = d~(u) + sum_{v in N+(u)} min(d~(u), d~(v)) when a plain count runs
+ * the shorter-list schedule (option "shorter", max d~ >= 64), else d~(u) + sum d~(v). */
 tc_status tc_partition(tc_graph *g, uint32_t world, uint32_t *bounds);
 
 /* a11.  NCCL plumbing (libnccl.so.2 is dlopen'ed; TC_ERR_NCCL if absent).

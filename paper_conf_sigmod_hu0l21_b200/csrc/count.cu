@@ -344,7 +344,8 @@ __global__ void edge_map_kernel(const uint64_t *__restrict__ offs, const uint32_
 
 // --------------------------------------------------------------- work model / analysis
 // w(u) = d~(u) + Σ_{v ∈ N+(u)} d~(v); sectors: 32-B sectors the Hu pattern touches with no reuse.
-// w[u] = d~(u) + Σ_{v ∈ N+(u)} d~(v) (the partition work model); sectors: the count's
+// w[u] = d~(u) + Σ_{v ∈ N+(u)} d~(v), with `shorter` Σ min(d~(u), d~(v)) (the partition
+// work model of the schedule that runs: the elements streamed per edge); sectors: the count's
 // algorithmic DRAM sectors with no reuse: per source with d~ >= 2 its
 // staged list + 1, per edge the streamed list + its offs pair — N+(v) (Hu's pattern), or
 // with `shorter` the shorter of N+(u), N+(v) (the shorter-list schedule of count_graph).
@@ -358,8 +359,8 @@ __global__ void work_kernel(const uint64_t *__restrict__ offs, const uint32_t *_
     for (uint64_t p = a + lane_id(); p < e; p += 32) {
       uint32_t v = col[p];
       uint64_t vb = offs[v], ve = offs[v + 1];
-      s += ve - vb;
       const bool own_u = shorter && ve - vb > e - a;  // E2: N+(u) is the streamed list
+      s += own_u ? e - a : ve - vb;                   // elements streamed for this edge
       const uint64_t sb = own_u ? a : vb, se = own_u ? e : ve, sx = own_u ? u : v;
       // streamed list span + its offs pair
       if (se > sb) sc += ((se * 4 - 1) >> 5) - ((sb * 4) >> 5) + 1;
@@ -862,6 +863,22 @@ void gather_per_vertex(Graph &g, const uint64_t *d_tnew, uint64_t *d_out) {
   TC_LAUNCH_CHECK();
 }
 
+// Does a plain count (count-only, bucketed) run the shorter-list schedule?  Option on, binary
+// search, and max d~ >= 64 (label-free: from ensure_od when it ran, else from the CSR).
+int shorter_schedule(Graph &g) {
+  if (!g_opt_shorter || g_opt_intersect != 0 || g.schedule == TC_SCHED_RANGE || g.schedule == TC_SCHED_EDGE_AORDER)
+    return 0;
+  uint32_t maxd = g.od_ready ? g.max_outdeg : 0;
+  if (!g.od_ready && g.n) {
+    DevBuf<uint32_t> od_new;
+    od_new.alloc(g.n, g.stream);
+    od_from_offs_kernel<<<grid_for(g.n, 256), 256, 0, g.stream>>>(g.offs.get(), g.n, od_new.get());
+    TC_LAUNCH_CHECK();
+    maxd = device_max_u32(od_new.get(), g.n, g.stream);
+  }
+  return maxd >= 64;
+}
+
 void partition_graph(Graph &g, uint32_t world, uint32_t *bounds) {
   cudaStream_t s = g.stream;
   const uint32_t n = g.n;
@@ -871,7 +888,8 @@ void partition_graph(Graph &g, uint32_t world, uint32_t *bounds) {
   pre.alloc((uint64_t)n + 1, s);
   db.alloc(world + 1, s);
   if (n) {
-    work_kernel<<<grid_for((uint64_t)n * 32, 256), 256, 0, s>>>(g.offs.get(), g.col.get(), n, w.get(), nullptr, 0);
+    work_kernel<<<grid_for((uint64_t)n * 32, 256), 256, 0, s>>>(g.offs.get(), g.col.get(), n, w.get(), nullptr,
+                                                                shorter_schedule(g));
     TC_LAUNCH_CHECK();
   }
   scan_u64(w.get(), pre.get(), n, s);
@@ -891,12 +909,7 @@ void analyze_graph(Graph &g) {
   sec.alloc(1, s);
   TC_CUDA(cudaMemsetAsync(sec.get(), 0, 8, s));
   if (n) {
-    // the schedule count_graph runs for a plain count: shorter-list when max d~ >= 64
-    DevBuf<uint32_t> od_new;
-    od_new.alloc(n, s);
-    od_from_offs_kernel<<<grid_for(n, 256), 256, 0, s>>>(g.offs.get(), n, od_new.get());
-    TC_LAUNCH_CHECK();
-    const int shorter = g_opt_shorter && g_opt_intersect == 0 && device_max_u32(od_new.get(), n, s) >= 64;
+    const int shorter = shorter_schedule(g);  // the schedule a plain count runs
     g.alg_model_shorter = shorter;
     work_kernel<<<grid_for((uint64_t)n * 32, 256), 256, 0, s>>>(g.offs.get(), g.col.get(), n, w.get(), sec.get(),
                                                                 shorter);

@@ -119,6 +119,7 @@ uint64_t count_graph(Graph &g, uint32_t u_begin, uint32_t u_end, uint64_t *d_tv 
 void map_edges_canonical(Graph &g, const uint64_t *d_te, uint64_t *d_out);
 void gather_per_vertex(Graph &g, const uint64_t *d_tnew, uint64_t *d_out);
 void partition_graph(Graph &g, uint32_t world, uint32_t *bounds);
+int shorter_schedule(Graph &g);  // a plain count runs the shorter-list schedule
 void analyze_graph(Graph &g);
 void build_units(Graph &g);  // edge-unit A-order buckets (count.cu)
 

@@ -1,8 +1,9 @@
 """World-size-2 tests of the N>1 host path on CPU (gloo): unique-id rendezvous,
 max-over-ranks timing, and the slice-then-sum exchange (a11) with the oracle standing in
 for the per-rank GPU partials.  The work-balanced bounds rule is restated here
-(w(u) = d~(u) + Σ_{v∈N+(u)} d~(v), bound g = first u with prefix >= g·W/world) and
-checked against the GPU implementation in tests/test_gpu_configs.py."""
+(w(u) = d~(u) + Σ_{v∈N+(u)} d~(v), or Σ min(d~(u), d~(v)) under the shorter-list schedule;
+bound g = first u with prefix >= g·W/world) and checked against the GPU implementation in
+tests/test_gpu_configs.py."""
 import os
 import socket
 
@@ -20,12 +21,13 @@ def _free_port():
     return p
 
 
-def work_bounds(offs, col, world, bucket_off=None):
+def work_bounds(offs, col, world, bucket_off=None, shorter=False):
     n = len(offs) - 1
     od = np.diff(offs.astype(np.int64))
     w = od.copy()
     for u in range(n):
-        w[u] += od[col[offs[u]:offs[u + 1]]].sum()
+        dv = od[col[offs[u]:offs[u + 1]]]
+        w[u] += np.minimum(dv, od[u]).sum() if shorter else dv.sum()
     pre = np.concatenate([[0], np.cumsum(w)])
     W = pre[-1]
     b = [0]
@@ -89,8 +91,8 @@ def test_bounds_rule_properties():
     spec = graphgen.rmat_spec(10, 16, 7)
     src, dst = graphgen.generate_cpu(spec)
     res = oracle.run(src, dst, spec.n, "degree", "none")
-    for world in (1, 2, 3, 8):
-        b = work_bounds(res["offs"], res["col"], world)
+    for world, shorter in ((1, False), (2, True), (3, False), (8, True)):
+        b = work_bounds(res["offs"], res["col"], world, shorter=shorter)
         assert b[0] == 0 and b[-1] == spec.n and all(x <= y for x, y in zip(b, b[1:]))
         parts = [oracle.count_forward(res["offs"], res["col"], b[i], b[i + 1]) for i in range(world)]
         assert sum(parts) == res["T"]

@@ -149,8 +149,8 @@ def test_config3_rmat_s22_ranges_partition_support():
         a = int(a)
         assert g.count_range(a, a + 40000) == oracle.count_forward(offs, col, a, a + 40000)
     # work-balanced partition = the restated rule (tests/test_dist_gloo.py)
-    for world in (2, 4, 8):
-        assert g.partition(world).tolist() == work_bounds_fast(offs, col, world)
+    for world in (2, 4, 8):  # max d~ >= 64: the shorter-list work model
+        assert g.partition(world).tolist() == work_bounds_fast(offs, col, world, shorter=True)
     # per-edge support (f1): Σ = 3T, and uniformly sampled edges (chosen without looking at
     # the GPU output) against the oracle's common-neighbour merge
     Te, te = g.count_edges()
@@ -160,11 +160,14 @@ def test_config3_rmat_s22_ranges_partition_support():
     g.free()
 
 
-def work_bounds_fast(offs, col, world):
+def work_bounds_fast(offs, col, world, shorter=False):
     od = np.diff(offs.astype(np.int64))
     s = np.zeros(len(od), np.int64)
     nz = od > 0
-    s[nz] = np.add.reduceat(od[col.astype(np.int64)], offs[:-1][nz].astype(np.int64))
+    dv = od[col.astype(np.int64)]
+    if shorter:  # the shorter-list schedule streams min(d~(u), d~(v)) per edge
+        dv = np.minimum(dv, np.repeat(od, od))
+    s[nz] = np.add.reduceat(dv, offs[:-1][nz].astype(np.int64))
     pre = np.concatenate([[0], np.cumsum(od + s)])
     n = len(od)
     b = [0] + [int(np.searchsorted(pre, (int(pre[-1]) * g) // world, side="left")) for g in range(1, world)] + [n]
@@ -176,4 +179,6 @@ def test_work_bounds_fast_matches_rule():
     src, dst = graphgen.generate_cpu(spec)
     res = oracle.run(src, dst, spec.n, "degree", "none")
     for w in (2, 3, 8):
-        assert work_bounds_fast(res["offs"], res["col"], w) == work_bounds(res["offs"], res["col"], w)
+        for sh in (False, True):
+            assert work_bounds_fast(res["offs"], res["col"], w, sh) == work_bounds(res["offs"], res["col"], w,
+                                                                                   shorter=sh)

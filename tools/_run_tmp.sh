@@ -1,5 +1,4 @@
 set -u
-OUT=gpurun_out; mkdir -p $OUT
-TAG=r02j STEPS="tests bench launches full" bash tools/gpu_round.sh
-for c in 3 2 1 5; do timeout 900 python bench.py --config $c --no-cpu-baseline --steps 5 --warmup 3 > $OUT/r02j_bench_cfg$c.json 2>&1; python -c "
-import json; d=json.load(open('$OUT/r02j_bench_cfg$c.json')); print($c, d['value'], d['count_ms'], d['whole_path']['value'], d['e2e']['value'], d['stages_ms'])"; done
+g++ -O3 -std=c++17 -pthread -Iinclude tools/aorder_bench.cpp -o /tmp/ab_new && g++ -O3 -std=c++17 -pthread -Iinclude -Itools tools/_aorder_bench_prev.cpp -o /tmp/ab_prev && python tools/dump_od.py 4 degree /tmp/od4.u32
+nproc; uptime
+for i in 1 2 3; do echo new; TC_AORDER_TRACE=1 /tmp/ab_new /tmp/od4.u32 3 2>&1 | grep aorder | tail -2; echo prev; TC_AORDER_TRACE=1 /tmp/ab_prev /tmp/od4.u32 3 2>&1 | grep aorder | tail -2; done
