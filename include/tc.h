@@ -230,7 +230,12 @@ tc_status tc_export_units(tc_graph *g, uint64_t *units, uint32_t *unit_off);
  * all edges that search it — SURVEY.md §8(a) a9 "the shorter of the two lists per edge ...
  * probed into the longer list"; 0 = always stream N+(v) against the staged N+(u), Hu's
  * pattern), "owner_span" / "owner_lspan" (streamed lists per warp / CTA work item of
- * that schedule, defaults 128 / 2048). */
+ * that schedule, defaults 128 / 2048), "otiles" (0 = auto, 1 = off (default), 2..255: the CTA work
+ * items of that schedule run in this many owner-label tiles — the owners of each long
+ * staged list grouped by the label tile of the owner, items listed tile by tile, so the
+ * lists streamed at any moment lie in one tile of col and are re-read from L2 instead of
+ * HBM; auto = ceil(col bytes / "otile_mb" MB), default 48), "otile_min" (a long list is
+ * tiled when it has >= otile_min x tiles owners, default 4). */
 tc_status tc_set_option(const char *key, int64_t value);
 
 /* Per-kernel profile since the last reset, as JSON text into buf (host, cap bytes):

@@ -206,6 +206,15 @@ tc_status tc_set_option(const char *key, int64_t value) {
     } else if (k == "owner_lspan") {
       TC_REQUIRE(value >= 8 && value <= (1 << 24), ST_INVALID, "owner_lspan: 8 .. 2^24");
       g_opt_owner_lspan = (int)value;
+    } else if (k == "otiles") {
+      TC_REQUIRE(value >= 0 && value <= 255, ST_INVALID, "otiles: 0 (auto) .. 255");
+      g_opt_otiles = (int)value;
+    } else if (k == "otile_mb") {
+      TC_REQUIRE(value >= 1 && value <= 4096, ST_INVALID, "otile_mb: 1 .. 4096");
+      g_opt_otile_mb = (int)value;
+    } else if (k == "otile_min") {
+      TC_REQUIRE(value >= 0 && value <= 1 << 20, ST_INVALID, "otile_min: 0 .. 2^20");
+      g_opt_otile_min = (int)value;
     }
     else if (k == "small_cap") {
       TC_REQUIRE(value >= 32 && value <= 2048 && (value & (value - 1)) == 0, ST_INVALID,

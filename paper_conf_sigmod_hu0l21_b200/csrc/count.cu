@@ -42,6 +42,9 @@ int g_opt_shorter = 1;       // count modes: per edge the shorter list is stream
 int g_opt_owner_span = 128;  // owners per warp item (shorter-list schedule)
 int g_opt_owner_lspan = 2048;  // owners per CTA item
 int g_opt_vtiles = 1;        // classic count: streamed lists in this many L2 label tiles (1 = off)
+int g_opt_otiles = 1;        // shorter-list CTA items: owner-label L2 tiles (0 = auto, 1 = off; default off: measured no faster)
+int g_opt_otile_mb = 48;     // auto: MB of col per owner-label tile
+int g_opt_otile_min = 4;     // a large x is tiled when it has >= otile_min * tiles owners
 
 using namespace cnt;
 namespace {
@@ -54,6 +57,7 @@ __global__ void items_hist_kernel(const uint64_t *__restrict__ offs, uint32_t ub
   for (uint64_t u = (uint64_t)ub + blockIdx.x * blockDim.x + threadIdx.x; u < ue; u += (uint64_t)gridDim.x * blockDim.x) {
     uint32_t d = (uint32_t)(offs[u + 1] - offs[u]);
     uint32_t it = items_of(d, owner_count(ow, (uint32_t)u, d), cap, ow);
+    if (ow.nt && d >= cap && ow.lg[u] != 0xffffffffu) it = 0;  // tiled x: its own item list
     if (it) atomicAdd(&s_h[deg_bin(d)], (unsigned long long)it);
   }
   __syncthreads();
@@ -84,6 +88,7 @@ __global__ __launch_bounds__(256) void items_scatter_kernel(const uint64_t *__re
       uint64_t u = c0 + (uint64_t)i * 256 + threadIdx.x;
       d[i] = u < ue ? (uint32_t)(offs[u + 1] - offs[u]) : 0u;
       it[i] = u < ue ? items_of(d[i], owner_count(ow, (uint32_t)u, d[i]), cap, ow) : 0u;
+      if (it[i] && ow.nt && d[i] >= cap && ow.lg[u] != 0xffffffffu) it[i] = 0;  // tiled x
       off[i] = it[i] ? atomicAdd(&s_cnt[deg_bin(d[i])], it[i]) : 0u;
     }
     __syncthreads();
@@ -109,14 +114,76 @@ __global__ void od_from_offs_kernel(const uint64_t *__restrict__ offs, uint32_t 
 // e1c[u] = #{v in N+(u): 1 <= d~(v) <= d~(u)} (u streams nothing, v's lists are searched in
 // N+(u)); e2c[v] += 1 for every u->v with d~(u) < d~(v) (u's list searched in N+(v)).
 // Sources with d~(u) < 2 close no triangle.
+// Owner-label tiles (option "otiles"): tile t = labels [bnd[t], bnd[t+1]), equal shares of
+// col; tile_of = the largest t with bnd[t] <= o (bnd staged in shared memory).
+constexpr uint32_t MAX_OTILES = 255;
+__device__ __forceinline__ uint32_t tile_of(const uint32_t *sb, uint32_t nt, uint32_t o) {
+  uint32_t lo = 0, len = nt;
+  while (len > 1) {
+    const uint32_t h = len >> 1;
+    lo = sb[lo + h] <= o ? lo + h : lo;
+    len -= h;
+  }
+  return lo;
+}
+__device__ __forceinline__ void stage_bounds(uint32_t *sb, const uint32_t *bnd, uint32_t nt) {
+  for (uint32_t t = threadIdx.x; t <= nt; t += blockDim.x) sb[t] = bnd ? bnd[t] : 0u;
+  __syncthreads();
+}
+// per lane: add 1 at row[key] for every lane with the same key (one atomic per distinct key)
+__device__ __forceinline__ uint32_t warp_agg_add(bool on, uint32_t key, uint32_t *row) {
+  const unsigned peers = __match_any_sync(0xffffffffu, on ? key : 0xffffffffu);
+  uint32_t base = 0;
+  const int leader = __ffs(peers) - 1;
+  if (on && (int)lane_id() == leader) base = atomicAdd(&row[key], (uint32_t)__popc(peers));
+  base = __shfl_sync(0xffffffffu, base, leader);
+  return base + __popc(peers & ((1u << lane_id()) - 1u));
+}
+__global__ void tile_bounds_kernel(const uint64_t *__restrict__ offs, uint32_t n, uint64_t m, uint32_t nt,
+                                   uint32_t *__restrict__ bnd) {
+  const uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
+  if (t > nt) return;
+  if (t == 0 || t == nt) {
+    bnd[t] = t ? n : 0u;
+    return;
+  }
+  const uint64_t target = m * t / nt;
+  uint32_t lo = 0, hi = n;  // first label o with offs[o] >= target
+  while (lo < hi) {
+    const uint32_t mid = lo + (hi - lo) / 2;
+    if (offs[mid] < target) lo = mid + 1;
+    else hi = mid;
+  }
+  bnd[t] = lo;
+}
+// lg[x] = index of x among the sources with d~(x) >= cap (large), else ~0
+__global__ void large_flag_kernel(const uint32_t *__restrict__ od, uint32_t n, uint32_t cap, uint32_t *__restrict__ f) {
+  for (uint64_t x = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; x < n; x += (uint64_t)gridDim.x * blockDim.x)
+    f[x] = od[x] >= cap ? 1u : 0u;
+}
+__global__ void large_index_kernel(const uint32_t *__restrict__ od, const uint64_t *__restrict__ pre, uint32_t n,
+                                   uint32_t cap, uint32_t *__restrict__ lg) {
+  for (uint64_t x = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; x < n; x += (uint64_t)gridDim.x * blockDim.x)
+    lg[x] = od[x] >= cap ? (uint32_t)pre[x] : 0xffffffffu;
+}
+
+// e1c[u] = #{v in N+(u): 1 <= d~(v) <= d~(u)} (u streams nothing, v's lists are searched in
+// N+(u)); e2c[v] += 1 for every u->v with d~(u) < d~(v) (u's list searched in N+(v)).
+// Sources with d~(u) < 2 close no triangle.  Owner tiles (tcnt != nullptr): also
+// tcnt[lg[x]*nt + tile(o)] += 1 for every owner o of a large x.
 __global__ void owners_count_kernel(const uint64_t *__restrict__ offs, const uint32_t *__restrict__ col,
                                     const uint32_t *__restrict__ od, uint32_t ub, uint32_t ue,
-                                    uint32_t *__restrict__ e1c, uint32_t *__restrict__ e2c) {
+                                    uint32_t *__restrict__ e1c, uint32_t *__restrict__ e2c,
+                                    const uint32_t *__restrict__ lg, const uint32_t *__restrict__ bnd, uint32_t nt,
+                                    uint32_t *__restrict__ tcnt) {
+  __shared__ uint32_t s_bnd[MAX_OTILES + 1];
+  if (tcnt) stage_bounds(s_bnd, bnd, nt);
   const uint64_t nw = (uint64_t)gridDim.x * (blockDim.x / 32);
   for (uint64_t u = ub + (uint64_t)blockIdx.x * (blockDim.x / 32) + warp_id(); u < ue; u += nw) {
     const uint64_t a = offs[u];
     const uint32_t du = (uint32_t)(offs[u + 1] - a);
     if (du < 2) continue;
+    const uint32_t lu = tcnt ? lg[u] : 0xffffffffu;  // warp-uniform
     uint32_t c1 = 0;
     for (uint32_t j0 = 0; j0 < du; j0 += 32) {
       const uint32_t j = j0 + lane_id();
@@ -125,10 +192,87 @@ __global__ void owners_count_kernel(const uint64_t *__restrict__ offs, const uin
         v = col[a + j];
         dv = od[v];
       }
-      c1 += __popc(__ballot_sync(0xffffffffu, j < du && dv >= 1 && dv <= du));
-      if (j < du && dv > du) atomicAdd(&e2c[v], 1u);
+      const bool e1 = j < du && dv >= 1 && dv <= du;
+      c1 += __popc(__ballot_sync(0xffffffffu, e1));
+      if (lu != 0xffffffffu) warp_agg_add(e1, e1 ? tile_of(s_bnd, nt, v) : 0u, tcnt + (uint64_t)lu * nt);
+      if (j < du && dv > du) {
+        atomicAdd(&e2c[v], 1u);
+        if (tcnt) {
+          const uint32_t lv = lg[v];
+          if (lv != 0xffffffffu) atomicAdd(&tcnt[(uint64_t)lv * nt + tile_of(s_bnd, nt, (uint32_t)u)], 1u);
+        }
+      }
     }
     if (lane_id() == 0) e1c[u] = c1;
+  }
+}
+// per large x: tiled iff it has >= tmin owners (else lg[x] = ~0: untiled); tiled rows get
+// toff (exclusive prefix of the tile counts, then the total) and tcnt becomes the row's
+// write cursor
+__global__ void tile_offsets_kernel(uint32_t n, uint32_t *__restrict__ lg, const uint64_t *__restrict__ ooff,
+                                    uint32_t nt, uint32_t tmin, uint32_t *__restrict__ tcnt,
+                                    uint32_t *__restrict__ toff) {
+  for (uint64_t x = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; x < n; x += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t l = lg[x];
+    if (l == 0xffffffffu) continue;
+    if (ooff[x + 1] - ooff[x] < tmin) {
+      lg[x] = 0xffffffffu;
+      continue;
+    }
+    uint32_t *c = tcnt + (uint64_t)l * nt, *o = toff + (uint64_t)l * (nt + 1);
+    uint32_t acc = 0;
+    for (uint32_t t = 0; t < nt; ++t) {
+      const uint32_t k = c[t];
+      o[t] = acc;
+      c[t] = acc;
+      acc += k;
+    }
+    o[nt] = acc;
+  }
+}
+// CTA items of the tiled x, tile by tile: per tile the item count, then cursors, then the
+// items (x << 32) | (t << 24) | chunk (ceil(owners in tile / lspan) chunks)
+__global__ void tile_items_count_kernel(uint32_t n, const uint32_t *__restrict__ lg, const uint32_t *__restrict__ toff,
+                                        uint32_t nt, uint32_t lspan, unsigned long long *__restrict__ tile_items) {
+  __shared__ unsigned long long s_c[MAX_OTILES];
+  for (uint32_t t = threadIdx.x; t < nt; t += blockDim.x) s_c[t] = 0;
+  __syncthreads();
+  for (uint64_t x = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; x < n; x += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t l = lg[x];
+    if (l == 0xffffffffu) continue;
+    const uint32_t *o = toff + (uint64_t)l * (nt + 1);
+    for (uint32_t t = 0; t < nt; ++t) {
+      const uint32_t k = o[t + 1] - o[t];
+      if (k) atomicAdd(&s_c[t], (unsigned long long)((k + lspan - 1) / lspan));
+    }
+  }
+  __syncthreads();
+  for (uint32_t t = threadIdx.x; t < nt; t += blockDim.x)
+    if (s_c[t]) atomicAdd(&tile_items[t], s_c[t]);
+}
+__global__ void tile_items_scan_kernel(unsigned long long *tile_items, uint32_t nt) {
+  // tile_items[0..nt) counts -> [nt .. 2nt) cursors, [2nt] total (one thread: nt <= 255)
+  unsigned long long acc = 0;
+  for (uint32_t t = 0; t < nt; ++t) {
+    tile_items[nt + t] = acc;
+    acc += tile_items[t];
+  }
+  tile_items[2 * nt] = acc;
+}
+__global__ void tile_items_scatter_kernel(uint32_t n, const uint32_t *__restrict__ lg,
+                                          const uint32_t *__restrict__ toff, uint32_t nt, uint32_t lspan,
+                                          unsigned long long *__restrict__ cursor, uint64_t *__restrict__ items) {
+  for (uint64_t x = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; x < n; x += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t l = lg[x];
+    if (l == 0xffffffffu) continue;
+    const uint32_t *o = toff + (uint64_t)l * (nt + 1);
+    for (uint32_t t = 0; t < nt; ++t) {
+      const uint32_t k = o[t + 1] - o[t];
+      if (!k) continue;
+      const uint32_t ni = (k + lspan - 1) / lspan;
+      const unsigned long long p = atomicAdd(&cursor[t], (unsigned long long)ni);
+      for (uint32_t c = 0; c < ni; ++c) items[p + c] = (x << 32) | ((uint64_t)t << 24) | c;
+    }
   }
 }
 __global__ void owners_total_kernel(const uint32_t *__restrict__ e1c, uint32_t n, uint32_t *__restrict__ c) {
@@ -141,17 +285,22 @@ __global__ void owners_cursor_kernel(const uint64_t *__restrict__ ooff, const ui
   for (uint64_t x = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; x < n; x += (uint64_t)gridDim.x * blockDim.x)
     cur[x] = ooff[x] + e1c[x];
 }
-// owners of x: its E1 out-neighbours (N+(x) order) then its E2 in-neighbours (any order)
+// owners of x: its E1 out-neighbours (N+(x) order) then its E2 in-neighbours (any order);
+// a tiled x (lg[x] != ~0, owner tiles on): grouped by owner tile through the row cursors
 __global__ void owners_scatter_kernel(const uint64_t *__restrict__ offs, const uint32_t *__restrict__ col,
                                       const uint32_t *__restrict__ od, uint32_t ub, uint32_t ue,
                                       const uint64_t *__restrict__ ooff, unsigned long long *__restrict__ e2cur,
-                                      uint32_t *__restrict__ own) {
+                                      uint32_t *__restrict__ own, const uint32_t *__restrict__ lg,
+                                      const uint32_t *__restrict__ bnd, uint32_t nt, uint32_t *__restrict__ tcur) {
+  __shared__ uint32_t s_bnd[MAX_OTILES + 1];
+  if (tcur) stage_bounds(s_bnd, bnd, nt);
   const uint64_t nw = (uint64_t)gridDim.x * (blockDim.x / 32);
   for (uint64_t u = ub + (uint64_t)blockIdx.x * (blockDim.x / 32) + warp_id(); u < ue; u += nw) {
     const uint64_t a = offs[u];
     const uint32_t du = (uint32_t)(offs[u + 1] - a);
     if (du < 2) continue;
     uint64_t p1 = ooff[u];
+    const uint32_t lu = tcur ? lg[u] : 0xffffffffu;  // warp-uniform
     for (uint32_t j0 = 0; j0 < du; j0 += 32) {
       const uint32_t j = j0 + lane_id();
       uint32_t v = 0, dv = 0;
@@ -160,10 +309,21 @@ __global__ void owners_scatter_kernel(const uint64_t *__restrict__ offs, const u
         dv = od[v];
       }
       const bool e1 = j < du && dv >= 1 && dv <= du;
-      const unsigned m1 = __ballot_sync(0xffffffffu, e1);
-      if (e1) own[p1 + __popc(m1 & ((1u << lane_id()) - 1u))] = v;
-      p1 += __popc(m1);
-      if (j < du && dv > du) own[atomicAdd(&e2cur[v], 1ull)] = (uint32_t)u;
+      if (lu != 0xffffffffu) {
+        const uint32_t r = warp_agg_add(e1, e1 ? tile_of(s_bnd, nt, v) : 0u, tcur + (uint64_t)lu * nt);
+        if (e1) own[p1 + r] = v;
+      } else {
+        const unsigned m1 = __ballot_sync(0xffffffffu, e1);
+        if (e1) own[p1 + __popc(m1 & ((1u << lane_id()) - 1u))] = v;
+        p1 += __popc(m1);
+      }
+      if (j < du && dv > du) {
+        const uint32_t lv = tcur ? lg[v] : 0xffffffffu;
+        if (lv != 0xffffffffu)
+          own[ooff[v] + atomicAdd(&tcur[(uint64_t)lv * nt + tile_of(s_bnd, nt, (uint32_t)u)], 1u)] = (uint32_t)u;
+        else
+          own[atomicAdd(&e2cur[v], 1ull)] = (uint32_t)u;
+      }
     }
   }
 }
@@ -638,6 +798,9 @@ uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *
       // streamed and searched in the longer one, which is staged once for all its owners
       Owners ow{nullptr, nullptr, 0, 0, 0, 0xffffffffu};
       DevBuf<uint32_t> od_new, e1c, e2c, own;
+      DevBuf<uint32_t> lg, bnd, tcnt, toff;  // owner tiles
+      uint32_t nt = 0;
+      uint64_t nlarge_x = 0;
       DevBuf<uint64_t> ooff;
       DevBuf<unsigned long long> e2cur;
       uint32_t iub = ub, iue = ue;  // sources of the item list
@@ -666,20 +829,63 @@ uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *
         ProfScope prof_owners("owners", s, 0.0);
         TC_CUDA(cudaMemsetAsync(e1c.get(), 0, e1c.bytes(), s));
         TC_CUDA(cudaMemsetAsync(e2c.get(), 0, e2c.bytes(), s));
+        // owner-label L2 tiles of the CTA items (option "otiles"): col cut into nt equal
+        // label tiles; the large x with enough owners get their owners grouped by tile
+        nt = g_opt_otiles == 1 ? 0u
+             : g_opt_otiles > 1 ? (uint32_t)g_opt_otiles
+                                : (uint32_t)((g.m * 4 + ((uint64_t)g_opt_otile_mb << 20) - 1) / ((uint64_t)g_opt_otile_mb << 20));
+        if (nt > MAX_OTILES) nt = MAX_OTILES;
+        if ((uint64_t)n / (uint64_t)g_opt_owner_lspan >= (1ull << 24)) nt = 0;  // chunk index in 24 bits
+        if (nt < 2) nt = 0;
+        if (nt) {
+          bnd.alloc(nt + 1, s);
+          tile_bounds_kernel<<<grid_for(nt + 1, 256), 256, 0, s>>>(g.offs.get(), n, g.m, nt, bnd.get());
+          TC_LAUNCH_CHECK();
+          lg.alloc(n, s);
+          DevBuf<uint64_t> lpre;
+          lpre.alloc((uint64_t)n + 1, s);
+          large_flag_kernel<<<grid_for(n, 256), 256, 0, s>>>(od_new.get(), n, cap, lg.get());
+          TC_LAUNCH_CHECK();
+          scan_u32_to_u64(lg.get(), lpre.get(), n, s);
+          large_index_kernel<<<grid_for(n, 256), 256, 0, s>>>(od_new.get(), lpre.get(), n, cap, lg.get());
+          TC_LAUNCH_CHECK();
+          uint64_t nL = 0;
+          TC_CUDA(cudaMemcpyAsync(&nL, lpre.get() + n, sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
+          TC_CUDA(cudaStreamSynchronize(s));
+          nlarge_x = nL;
+          tcnt.alloc(nL * nt + 1, s);
+          toff.alloc(nL * (nt + 1) + 1, s);
+          TC_CUDA(cudaMemsetAsync(tcnt.get(), 0, tcnt.bytes(), s));
+          nlaunch += 4;
+        }
         const unsigned wgrid = grid_for((uint64_t)(ue - ub) * 32, 256, 8);
         owners_count_kernel<<<wgrid, 256, 0, s>>>(g.offs.get(), g.col.get(), od_new.get(), ub, ue, e1c.get(),
-                                                  e2c.get());
+                                                  e2c.get(), lg.get(), bnd.get(), nt, nt ? tcnt.get() : nullptr);
         TC_LAUNCH_CHECK();
         owners_total_kernel<<<grid_for(n, 256), 256, 0, s>>>(e1c.get(), n, e2c.get());
         TC_LAUNCH_CHECK();
         scan_u32_to_u64(e2c.get(), ooff.get(), n, s);
         owners_cursor_kernel<<<grid_for(n, 256), 256, 0, s>>>(ooff.get(), e1c.get(), n, e2cur.get());
         TC_LAUNCH_CHECK();
+        if (nt) {
+          const uint64_t tmin = (uint64_t)g_opt_otile_min * nt;
+          tile_offsets_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, lg.get(), ooff.get(), nt,
+                                                               (uint32_t)std::min<uint64_t>(tmin, 0xffffffffu),
+                                                               tcnt.get(), toff.get());
+          TC_LAUNCH_CHECK();
+          ++nlaunch;
+        }
         owners_scatter_kernel<<<wgrid, 256, 0, s>>>(g.offs.get(), g.col.get(), od_new.get(), ub, ue, ooff.get(),
-                                                    e2cur.get(), own.get());
+                                                    e2cur.get(), own.get(), lg.get(), bnd.get(), nt,
+                                                    nt ? tcnt.get() : nullptr);
         TC_LAUNCH_CHECK();
         nlaunch += 6;
         ow = Owners{ooff.get(), own.get(), (uint32_t)g_opt_owner_span, (uint32_t)g_opt_owner_lspan, 0, 0xffffffffu};
+        if (nt) {
+          ow.lg = lg.get();
+          ow.toff = toff.get();
+          ow.nt = nt;
+        }
         iub = 0;  // an E2 edge u -> v is counted at v, any label
         iue = n;
       }
@@ -703,6 +909,25 @@ uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *
         TC_LAUNCH_CHECK();
         ++nlaunch;
       }
+      // CTA items of the tiled x, listed tile by tile ([2nt] total, [2nt+1] fetch counter)
+      DevBuf<unsigned long long> titems;
+      DevBuf<uint64_t> items_t;
+      uint64_t ntiled = 0;
+      if (nt) {
+        titems.alloc(2 * (uint64_t)nt + 2, s);
+        TC_CUDA(cudaMemsetAsync(titems.get(), 0, titems.bytes(), s));
+        tile_items_count_kernel<<<grid_for(g.n, 256, 4), 256, 0, s>>>(g.n, lg.get(), toff.get(), nt, ow.lspan,
+                                                                         titems.get());
+        TC_LAUNCH_CHECK();
+        tile_items_scan_kernel<<<1, 1, 0, s>>>(titems.get(), nt);
+        TC_LAUNCH_CHECK();
+        items_t.alloc(g.m / ow.lspan + nlarge_x * nt + 1, s);
+        tile_items_scatter_kernel<<<grid_for(g.n, 256, 4), 256, 0, s>>>(g.n, lg.get(), toff.get(), nt, ow.lspan,
+                                                                           titems.get() + nt, items_t.get());
+        TC_LAUNCH_CHECK();
+        TC_CUDA(cudaMemcpyAsync(&ntiled, titems.get() + 2 * nt, sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
+        nlaunch += 3;
+      }
       std::vector<unsigned long long> hh(32);
       TC_CUDA(cudaMemcpyAsync(hh.data(), hist.get(), 32 * sizeof(unsigned long long), cudaMemcpyDeviceToHost, s));
       TC_CUDA(cudaStreamSynchronize(s));
@@ -723,8 +948,19 @@ uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *
         }
       cap_small = fit_cap(cap_small, pv);
       nlaunch += 2;
-      if (nitems) {
+      if (nitems || ntiled) {
         if (kernel_ms) TC_CUDA(cudaEventRecord(e0, s));
+        if (ntiled) {
+          size_t smem = LG_SMEM_WORDS * sizeof(uint32_t);
+          const void *large_fn = large_kernel(0, true);
+          int occ = occupancy(large_fn, LG_THREADS, smem);
+          unsigned grid = (unsigned)std::min<uint64_t>(ntiled, (uint64_t)num_sms() * occ);
+          ProfScope prof("count_large", s, 0.0);
+          launch(large_fn, grid, LG_THREADS, smem, s, (const uint64_t *)g.offs.get(), (const uint32_t *)g.col.get(),
+                 (const uint64_t *)items_t.get(), ntiled, titems.get() + 2 * nt + 1, (unsigned long long *)dT.get(), tv,
+                 vbits, ow);
+          ++nlaunch;
+        }
         if (nlarge) {
           size_t smem = LG_SMEM_WORDS * sizeof(uint32_t);
           const void *large_fn = large_kernel(ow.own ? 0 : mode, ow.own != nullptr);

@@ -31,7 +31,13 @@ constexpr int TS_W = 2;               // warp items
 #ifndef TC_TS_L
 #define TC_TS_L 1
 #endif
-constexpr int TS_L = TC_TS_L;         // CTA items (pieces)
+constexpr int TS_L = TC_TS_L;         // CTA items (pieces): the table's size in smem
+// CTA items: the piece's table takes all the room left after the padded piece (a shorter
+// piece leaves more), up to 2^TS_LMAX buckets per element
+#ifndef TC_TS_LMAX
+#define TC_TS_LMAX 4
+#endif
+constexpr int TS_LMAX = TC_TS_LMAX;
 constexpr uint32_t LG_SMEM_WORDS = (PIECE + 72) + ((PIECE << TS_L) + 64) / 2;  // piece (+pad) + u16 table
 constexpr uint32_t CHUNK = 8;         // worklist entries per atomic fetch
 
@@ -55,6 +61,14 @@ struct Owners {
   // classic schedule, count modes: only v in [vlo, vhi) this pass (L2 tiles of the
   // streamed lists, option "vtiles"); [0, 2^32) = every v
   uint32_t vlo = 0, vhi = 0xffffffffu;
+  // CTA items in owner-label L2 tiles (option "otiles"; nt = 0: off).  The owners of a tiled
+  // x (lg[x] != ~0) are grouped by the label tile of the owner: tile t of x is
+  // own[off[x] + toff[lg[x]*(nt+1) + t] .. + toff[.. + t + 1]); its CTA items are
+  // (x << 32) | (t << 24) | chunk, listed tile by tile, so the lists streamed at any moment
+  // lie in one label tile (<= a few tens of MB of col) and are re-read from L2, not HBM
+  const uint32_t *lg = nullptr;
+  const uint32_t *toff = nullptr;
+  uint32_t nt = 0;
 };
 
 __device__ __forceinline__ uint32_t ldg_u32(const uint32_t *p) { return __ldg(p); }
@@ -668,8 +682,7 @@ __global__ __launch_bounds__(LG_THREADS, OWN ? TC_LG_MINB_OWN : 5) void count_la
                                                                  const uint64_t *__restrict__ items, uint64_t nitems,
                                                                  unsigned long long *ctr, unsigned long long *T,
                                                                  unsigned long long *tv, uint32_t vbits, Owners ow) {
-  uint32_t *s_piece = tc_smem;  // PIECE + 72 words (alignment slack + padding), then the table
-  constexpr uint32_t tbase_lg = PIECE + 72;
+  uint32_t *s_piece = tc_smem;  // the piece (alignment slack + padding), then the table
   __shared__ WarpScratch s_ws[LG_WARPS];
   __shared__ uint32_t s_red[LG_WARPS];
   __shared__ __align__(8) uint64_t s_bar;
@@ -687,12 +700,24 @@ __global__ __launch_bounds__(LG_THREADS, OWN ? TC_LG_MINB_OWN : 5) void count_la
     __syncthreads();
     if (item >= nitems) break;
     const uint64_t it = items[item];
-    const uint32_t u = (uint32_t)(it >> 32), cbeg = (uint32_t)it;
+    const uint32_t u = (uint32_t)(it >> 32);
+    uint32_t cbeg = (uint32_t)it;
     const uint64_t a = offs[u];
     const uint32_t L = (uint32_t)(offs[u + 1] - a);
-    // owners: N+(u) itself (classic) or the shorter-list owners of u (count modes)
+    // owners: N+(u) itself (classic) or the shorter-list owners of u (count modes), or
+    // one label tile of them (tiled x)
     const uint32_t *olist = OWN ? ow.own + ow.off[u] : col + a;
-    const uint32_t C = OWN ? (uint32_t)(ow.off[u + 1] - ow.off[u]) : L;
+    uint32_t C = OWN ? (uint32_t)(ow.off[u + 1] - ow.off[u]) : L;
+    if (OWN && ow.nt) {
+      const uint32_t l = ow.lg[u];
+      if (l != 0xffffffffu) {
+        const uint32_t *tt = ow.toff + (uint64_t)l * (ow.nt + 1) + ((uint32_t)(it >> 24) & 0xffu);
+        const uint32_t t0 = tt[0];
+        olist += t0;
+        C = tt[1] - t0;
+        cbeg = ((uint32_t)it & 0xffffffu) * ow.lspan;
+      }
+    }
     const uint32_t cend = min(C, cbeg + (OWN ? ow.lspan : LV));
     uint64_t ucnt = 0;
     for (uint32_t p0 = 0; p0 < L; p0 += PIECE) {
@@ -712,11 +737,13 @@ __global__ __launch_bounds__(LG_THREADS, OWN ? TC_LG_MINB_OWN : 5) void count_la
       if (threadIdx.x == 0) s_next = 0;  // published by the barrier below
       phase ^= 1u;
       const uint32_t *list = s_piece + shift;
-      {  // pad the piece with +inf up to a power of two (+64) for the fixed-depth search
-        const uint32_t P = (1u << ceil_log2(plen)) + 64;
-        for (uint32_t j = plen + threadIdx.x; j < P; j += LG_THREADS) s_piece[shift + j] = 0xffffffffu;
-        __syncthreads();
-      }
+      // pad the piece with +inf up to a power of two (+64) for the fixed-depth search; the
+      // bracket table starts right after it (u16 entries, 4-byte aligned)
+      const uint32_t P = (1u << ceil_log2(plen)) + 64;
+      for (uint32_t j = plen + threadIdx.x; j < P; j += LG_THREADS) s_piece[shift + j] = 0xffffffffu;
+      __syncthreads();
+      const uint32_t tbase = shift + P;
+      const uint32_t tcap = (LG_SMEM_WORDS - tbase) * 2u;  // table entries that fit
       const uint32_t lo = list[0], hi = list[plen - 1];
       // CTA-wide bracket table of the piece (shared by all warps of the item); absolute
       // (bucket w >> sh over [0, 2^vbits)) when the piece spans the whole label range
@@ -729,10 +756,12 @@ __global__ __launch_bounds__(LG_THREADS, OWN ? TC_LG_MINB_OWN : 5) void count_la
         abs_t = span_bits >= (int)vbits;
         const uint32_t tlo = abs_t ? 0u : lo;
         const uint32_t thi = abs_t ? (vbits >= 32 ? 0xffffffffu : (1u << vbits) - 1u) : hi;
-        const int tb = abs_t ? (int)vbits : span_bits;
-        sh = tb > S + TS_L ? (uint32_t)(tb - S - TS_L) : 0u;
+        // finest bucket width 2^sh whose table (entries 0 .. B, B = (span >> sh) + 1) fits in
+        // the room left, at most 2^TS_LMAX buckets per element (fewer search steps S2)
+        const uint32_t lim = min(tcap - 2u, 1u << (S + TS_LMAX));
+        while (((thi - tlo) >> sh) > lim) ++sh;
         const uint32_t B = ((thi - tlo) >> sh) + 1;
-        uint16_t *tab = reinterpret_cast<uint16_t *>(tc_smem + tbase_lg);
+        uint16_t *tab = reinterpret_cast<uint16_t *>(tc_smem + tbase);
         for (uint32_t j = threadIdx.x; j < plen; j += LG_THREADS) {
           const uint32_t bj = (list[j] - tlo) >> sh;
           const int bp = j ? (int)((list[j - 1] - tlo) >> sh) : -1;
@@ -763,7 +792,7 @@ __global__ __launch_bounds__(LG_THREADS, OWN ? TC_LG_MINB_OWN : 5) void count_la
         if (c0 >= cend) break;
         const bool valid = lane_id() < SUB && c0 + lane_id() < cend;
         const uint32_t v = valid ? ldg_u32(olist + c0 + lane_id()) : 0u;
-        cnt += warp_chunk<MODE, MODE == 0 ? 8 : 4>(offs, col, v, valid, list, shift, S2 >= 0 ? tbase_lg : 0xffffffffu, 0xffffffffu, plen,
+        cnt += warp_chunk<MODE, MODE == 0 ? 8 : 4>(offs, col, v, valid, list, shift, S2 >= 0 ? tbase : 0xffffffffu, 0xffffffffu, plen,
                                 true, lo, hi, ws, tv, c0 + lane_id(), a, a + p0, vbits, S2 >= 0 ? S2 : -2, sh,
                                 abs_t ? 1 : 0);
       }

@@ -489,6 +489,33 @@ def test_shorter_list_schedule(cap, spans):
         tc.tc_set_option("owner_lspan", 2048)
 
 
+@pytest.mark.parametrize("cap", [32, 256])
+def test_owner_tiles(cap):
+    """CTA items of the shorter-list schedule in owner-label L2 tiles (option otiles): every
+    tile count / tiling threshold / item span gives the oracle's T, whole and on slices."""
+    tc.tc_set_option("small_cap", cap)
+    try:
+        for seed, (sc, ef, d, r) in enumerate(((13, 32, "degree", "paper"), (12, 16, "paper", "none"),
+                                               (11, 48, "id", "degree"))):
+            spec = graphgen.rmat_spec(sc, ef, 950 + seed)
+            src, dst = graphgen.generate_cpu(spec)
+            ref = oracle.run(src, dst, spec.n, d, r)
+            g = tc.Graph(src, dst, spec.n).direct(d).reorder(r)
+            for nt, tmin, lspan in ((2, 0, 2048), (7, 0, 8), (7, 4, 64), (255, 0, 2048), (255, 1, 16)):
+                tc.tc_set_option("otiles", nt)
+                tc.tc_set_option("otile_min", tmin)
+                tc.tc_set_option("owner_lspan", lspan)
+                assert g.count() == ref["T"], (seed, nt, tmin, lspan)
+                b = g.partition(3).tolist()
+                assert sum(g.count_range(a, c) for a, c in zip(b, b[1:])) == ref["T"], (seed, nt, tmin, lspan)
+            g.free()
+    finally:
+        tc.tc_set_option("otiles", 1)
+        tc.tc_set_option("otile_min", 4)
+        tc.tc_set_option("owner_lspan", 2048)
+        tc.tc_set_option("small_cap", 256)
+
+
 def test_extra_compute_instrumented_kernel_counts_unchanged():
     """The §5.3 balance-point instrumentation (option extra_compute, MODE 3: p_c extra
     searches per wedge, results discarded) leaves T and t(v) equal to the oracle's."""

@@ -22,7 +22,11 @@ def main():
     ap.add_argument("--values", default="0,1")
     ap.add_argument("--rule", default="degree:none")
     ap.add_argument("--reps", type=int, default=5)
+    ap.add_argument("--set", default="", help="fixed options k=v,k=v applied first")
     a = ap.parse_args()
+    for kv in filter(None, a.set.split(",")):
+        k, v = kv.split("=")
+        tc.tc_set_option(k, int(v))
     spec = graphgen.CONFIGS[a.config]
     src = torch.empty(spec.samples, dtype=torch.int32, device="cuda")
     dst = torch.empty(spec.samples, dtype=torch.int32, device="cuda")
