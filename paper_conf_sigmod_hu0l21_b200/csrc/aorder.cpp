@@ -287,7 +287,7 @@ static unsigned host_threads(size_t n) {
 // ~10 B per unit otherwise cost as much as the greedy itself).  One A-order at a time.
 struct AOrderWorkspace {
   std::mutex mu;
-  std::vector<uint32_t> vmem, vcomp, bucket_of, rank_of;
+  std::vector<uint32_t> vmem, vcomp, bmem, bcomp, rmem, rcomp;  // bucket / rank of vmem[i], vcomp[i]
   std::vector<int64_t> smem, scomp;  // S of vmem[i] / vcomp[i]
 };
 static AOrderWorkspace &workspace() {
@@ -388,7 +388,9 @@ static void aorder_core(size_t n, SF S, AF active, uint32_t k, int order, uint32
   const size_t b = (nact + k - 1) / k;
   std::vector<int64_t> mem_sup(b, 0);        // line 1
   std::vector<uint32_t> fill(b, 0);
-  uint32_t *bucket_of = grow(W.bucket_of, n), *rank_of = grow(W.rank_of, n);  // insertion record
+  // insertion record per placement index (sequential writes; the relabel scatters them)
+  uint32_t *bmem = grow(W.bmem, nmem), *rmem = grow(W.rmem, nmem);
+  uint32_t *bcomp = grow(W.bcomp, ncomp), *rcomp = grow(W.rcomp, ncomp);
   const int ib = b > 1 ? 64 - __builtin_clzll((unsigned long long)(b - 1)) : 1;
   const long double bound = (long double)smax * (long double)k * 2.0L + 2.0L;  // |mem_sup| < k smax
   const bool packed = bound * (long double)(1ull << ib) < 9.0e18L;
@@ -405,36 +407,73 @@ static void aorder_core(size_t n, SF S, AF active, uint32_t k, int order, uint32
     MonoQueue q;
     std::vector<uint64_t> keys;
     keys.reserve(b);
+    // One phase of the greedy: unit i takes the bucket at the top of the queue and the
+    // bucket's key grows by inc[i] (packed units).  While no re-entered key is pending, the
+    // top is the next key of the sorted current bin, so a run of placements is a straight
+    // loop over that bin (a grown key lands in a later bin whenever the bin is narrower
+    // than the smallest increment); a key re-entering the current bin goes through the
+    // queue's small heap and the step-by-step path.  full(pk) records a bucket that left.
+    auto phase = [&](size_t nu, auto inc, uint32_t *brec, uint32_t *rrec, auto full) {
+      size_t i = 0;
+      while (i < nu) {
+        if (q.heap.empty() && q.rpos < q.run.size()) {
+          const uint64_t *rp = q.run.data();
+          const size_t jend = std::min(q.run.size(), q.rpos + (nu - i));
+          size_t j = q.rpos;
+          bool reentered = false;
+          for (; j < jend; ++j, ++i) {
+            const uint64_t pk = rp[j];
+            const size_t bk = (size_t)(pk & imask);
+            const uint32_t r = fill[bk]++;
+            brec[i] = (uint32_t)bk;
+            rrec[i] = r;
+            const uint64_t npk = pk + inc(i);
+            if (r + 1 < k) {
+              const size_t bi = q.bin_of(npk);
+              if (bi == q.cur) {
+                q.push(npk);
+                reentered = true;
+                ++j;
+                ++i;
+                break;
+              }
+              q.bins[bi].push_back(npk);
+            } else {
+              full(bk, npk);
+            }
+          }
+          q.rpos = j;
+          if (!reentered) q.refill();
+          continue;
+        }
+        const uint64_t pk = q.top();
+        const size_t bk = (size_t)(pk & imask);
+        const uint32_t r = fill[bk]++;
+        brec[i] = (uint32_t)bk;
+        rrec[i] = r;
+        const uint64_t npk = pk + inc(i);
+        const bool live = r + 1 < k;
+        if (!live) full(bk, npk);
+        q.replace_top(npk, live);
+        ++i;
+      }
+    };
     for (size_t i = 0; i < b; ++i) keys.push_back(pack(i, 0, false));
     q.build(keys, max_pk, smin1 == INT64_MAX ? 0 : (uint64_t)smin1 << ib, ib);  // line 2: min queue
-    for (size_t i = 0; i < nmem; ++i) {          // line 5
-      const uint64_t pk = q.top();
-      const size_t bk = (size_t)(pk & imask);    // line 6
-      const uint32_t r = fill[bk]++;
-      bucket_of[vmem[i]] = (uint32_t)bk;        // line 7
-      rank_of[vmem[i]] = r;
-      const uint64_t npk = pk + ((uint64_t)smem[i] << ib);  // line 8: mem_sup += S(v)
-      const bool live = r + 1 < k;
-      if (!live) mem_sup[bk] = (int64_t)(npk >> ib) - off;
-      q.replace_top(npk, live);                  // line 9
-    }
+    // lines 5-9: memory-dominated v -> min bucket (line 6-7), mem_sup += S(v) (line 8), re-queue (line 9)
+    phase(
+        nmem, [&](size_t i) { return (uint64_t)smem[i] << ib; }, bmem, rmem,
+        [&](size_t bk, uint64_t npk) { mem_sup[bk] = (int64_t)(npk >> ib) - off; });
     q.for_each([&](uint64_t pk) { mem_sup[pk & imask] = (int64_t)(pk >> ib) - off; });
     if (trace_on()) t2 = now_ms();
     keys.clear();
     for (size_t i = 0; i < b; ++i)
       if (fill[i] < k) keys.push_back(pack(i, mem_sup[i], true));
     q.build(keys, max_pk, smin2 == INT64_MAX ? 0 : (uint64_t)smin2 << ib, ib);  // line 10: max queue
-    for (size_t i = 0; i < ncomp; ++i) {         // line 11
-      const uint64_t pk = q.top();
-      const size_t bk = (size_t)(pk & imask);    // line 12
-      const uint32_t r = fill[bk]++;
-      bucket_of[vcomp[i]] = (uint32_t)bk;       // line 13
-      rank_of[vcomp[i]] = r;
-      const uint64_t npk = pk + ((uint64_t)(-scomp[i]) << ib);  // line 14: mem_sup += S(v) <= 0
-      const bool live = r + 1 < k;
-      if (!live) mem_sup[bk] = off - (int64_t)(npk >> ib);
-      q.replace_top(npk, live);                  // line 15
-    }
+    // lines 11-15: computing-dominated v -> max bucket, mem_sup += S(v) <= 0 (its negated key grows)
+    phase(
+        ncomp, [&](size_t i) { return (uint64_t)(-scomp[i]) << ib; }, bcomp, rcomp,
+        [&](size_t bk, uint64_t npk) { mem_sup[bk] = off - (int64_t)(npk >> ib); });
     q.for_each([&](uint64_t pk) { mem_sup[pk & imask] = off - (int64_t)(pk >> ib); });
   } else if (b) {
     // generic tournament tree (mem_sup beyond the packed range)
@@ -444,8 +483,8 @@ static void aorder_core(size_t n, SF S, AF active, uint32_t k, int order, uint32
     q.build(b, mem_sup, alive);
     for (size_t i = 0; i < nmem; ++i) {          // line 5
       const int64_t bk = q.top();                // line 6
-      bucket_of[vmem[i]] = (uint32_t)bk;        // line 7
-      rank_of[vmem[i]] = fill[bk]++;
+      bmem[i] = (uint32_t)bk;                    // line 7
+      rmem[i] = fill[bk]++;
       mem_sup[bk] += smem[i];                    // line 8
       if (fill[bk] == k) alive[bk] = 0;
       q.update((size_t)bk, mem_sup[bk], alive[bk]);  // line 9
@@ -454,8 +493,8 @@ static void aorder_core(size_t n, SF S, AF active, uint32_t k, int order, uint32
     q.build(b, mem_sup, alive);
     for (size_t i = 0; i < ncomp; ++i) {         // line 11
       const int64_t bk = q.top();                // line 12
-      bucket_of[vcomp[i]] = (uint32_t)bk;       // line 13
-      rank_of[vcomp[i]] = fill[bk]++;
+      bcomp[i] = (uint32_t)bk;                   // line 13
+      rcomp[i] = fill[bk]++;
       mem_sup[bk] += scomp[i];                   // line 14
       if (fill[bk] == k) alive[bk] = 0;
       q.update((size_t)bk, mem_sup[bk], alive[bk]);  // line 15
@@ -471,9 +510,16 @@ static void aorder_core(size_t n, SF S, AF active, uint32_t k, int order, uint32
     eq3 += std::llabs(mem_sup[i]);           // Eq.3 objective (λ folded into S)
   }
   const uint32_t inactive0 = bucket_off[b];
+  par_chunks(nmem, T, [&](size_t lo, size_t hi, unsigned) {
+    for (size_t i = lo; i < hi; ++i) perm[vmem[i]] = bucket_off[bmem[i]] + rmem[i];
+  });
+  par_chunks(ncomp, T, [&](size_t lo, size_t hi, unsigned) {
+    for (size_t i = lo; i < hi; ++i) perm[vcomp[i]] = bucket_off[bcomp[i]] + rcomp[i];
+  });
   par_chunks(n, T, [&](size_t lo, size_t hi, unsigned t) {
     uint32_t idx = inactive0 + (uint32_t)ci[t];
-    for (size_t v = lo; v < hi; ++v) perm[v] = active(v) ? bucket_off[bucket_of[v]] + rank_of[v] : idx++;
+    for (size_t v = lo; v < hi; ++v)
+      if (!active(v)) perm[v] = idx++;
   });
   if (trace_on())
     fprintf(stderr, "aorder n=%zu mem=%zu comp=%zu b=%zu: classify %.1f ms, phase1 %.1f, phase2 %.1f, relabel %.1f\n",

@@ -280,11 +280,23 @@ __device__ __forceinline__ void fast_block(const uint32_t *__restrict__ p, const
                                            uint32_t &cnt) {
   uint32_t w[N];
 #pragma unroll
-  for (int k = 0; k < N; ++k) w[k] = ldg_u32(p + 32 * k);
+  for (int k = 0; k < N; ++k) {
+#ifdef TC_EXP_NOLOAD  // decomposition experiment: searches without the gather (T is wrong)
+    w[k] = (uint32_t)(((uintptr_t)(p + 32 * k) >> 2) * 2654435761u) >> 8;
+#else
+    w[k] = ldg_u32(p + 32 * k);
+#endif
+  }
 #pragma unroll
   for (int k = 0; k < N; ++k) {
     uint32_t pos;
+#ifdef TC_EXP_NOSEARCH  // decomposition experiment: gathers without the search (T is wrong)
+    const bool hit = w[k] == 0x7fffffffu;
+    pos = 0;
+    (void)search;
+#else
     const bool hit = search(w[k], pos);
+#endif
     cnt += hit ? 1u : 0u;
     if (MODE == 3) {  // §5.3 balance-point experiment, as in wedge_block
       uint32_t acc = 0;

@@ -36,7 +36,8 @@ def case(spec, d, r, sched=None, opts=(), per_vertex=True, per_edge=False):
     finally:
         for k, _ in opts:
             tc.tc_set_option(k, {"small_cap": 256, "shorter": 1, "intersect": 0, "peel_coop": 1,
-                                 "owner_span": 128, "owner_lspan": 2048, "extra_compute": -1}[k])
+                                 "owner_span": 128, "owner_lspan": 2048, "extra_compute": -1,
+                                 "otiles": 1, "otile_min": 4}[k])
     print("ok", spec.name, d, r, sched, opts, flush=True)
 
 
@@ -79,6 +80,8 @@ def main():
     case(s10, "degree", "none", opts=(("intersect", 2),), per_vertex=False)       # bitmap
     case(s11, "paper", "none", opts=(("peel_coop", 0),))                          # multi-launch peel
     case(s10, "degree", "none", opts=(("extra_compute", 8), ("shorter", 0)))      # §5.3 instrumented
+    case(s11, "degree", "paper", opts=(("small_cap", 32), ("otiles", 7), ("otile_min", 0), ("owner_lspan", 8)),
+         per_vertex=False)                                                          # owner-label tiles
     print("all sanitizer cases passed")
 
 
