@@ -235,7 +235,11 @@ tc_status tc_export_units(tc_graph *g, uint64_t *units, uint32_t *unit_off);
  * staged list grouped by the label tile of the owner, items listed tile by tile, so the
  * lists streamed at any moment lie in one tile of col and are re-read from L2 instead of
  * HBM; auto = ceil(col bytes / "otile_mb" MB), default 48), "otile_min" (a long list is
- * tiled when it has >= otile_min x tiles owners, default 4). */
+ * tiled when it has >= otile_min x tiles owners, default 4), "cuckoo" (count-only CTA work
+ * items: the staged list is held as a cuckoo hash set — two tables of 2^b slots, probe =
+ * two independent shared loads — instead of the sorted piece with its bracket table; the
+ * value is the eviction limit per insertion, default 64, 0 = off; an insertion that fails
+ * falls back to the sorted piece, counts are unchanged). */
 tc_status tc_set_option(const char *key, int64_t value);
 
 /* Per-kernel profile since the last reset, as JSON text into buf (host, cap bytes):

@@ -206,6 +206,9 @@ tc_status tc_set_option(const char *key, int64_t value) {
     } else if (k == "owner_lspan") {
       TC_REQUIRE(value >= 8 && value <= (1 << 24), ST_INVALID, "owner_lspan: 8 .. 2^24");
       g_opt_owner_lspan = (int)value;
+    } else if (k == "cuckoo") {
+      TC_REQUIRE(value >= 0 && value <= 1024, ST_INVALID, "cuckoo: 0 (off) .. 1024 evictions");
+      g_opt_cuckoo = (int)value;
     } else if (k == "otiles") {
       TC_REQUIRE(value >= 0 && value <= 255, ST_INVALID, "otiles: 0 (auto) .. 255");
       g_opt_otiles = (int)value;

@@ -42,6 +42,7 @@ int g_opt_shorter = 1;       // count modes: per edge the shorter list is stream
 int g_opt_owner_span = 128;  // owners per warp item (shorter-list schedule)
 int g_opt_owner_lspan = 2048;  // owners per CTA item
 int g_opt_vtiles = 1;        // classic count: streamed lists in this many L2 label tiles (1 = off)
+int g_opt_cuckoo = 64;       // count-only CTA items: cuckoo set of the staged piece, max evictions (0 = off)
 int g_opt_otiles = 1;        // shorter-list CTA items: owner-label L2 tiles (0 = auto, 1 = off; default off: measured no faster)
 int g_opt_otile_mb = 48;     // auto: MB of col per owner-label tile
 int g_opt_otile_min = 4;     // a large x is tiled when it has >= otile_min * tiles owners
@@ -560,7 +561,7 @@ __global__ void bounds_kernel(const uint64_t *__restrict__ pre, uint32_t n, uint
 static std::mutex g_cfg_mu;
 struct DeviceCfg {
   bool configured = false;
-  int bracket = 1, intersect = 0, extra = -1;
+  int bracket = 1, intersect = 0, extra = -1, cuckoo = 64;
 };
 static DeviceCfg g_cfg[64];
 
@@ -596,9 +597,10 @@ static void configure_kernels() {
   DeviceCfg &c = device_cfg();
   configure_kernels_locked(c);
   const int extra = g_opt_extra >= 0 ? g_opt_extra : c.extra;
-  if (g_opt_bracket != c.bracket || g_opt_intersect != c.intersect || extra != c.extra) {
-    small_set_constants(g_opt_bracket, g_opt_intersect, extra < 0 ? 0 : extra);
-    large_set_constants(g_opt_bracket, g_opt_intersect, extra < 0 ? 0 : extra);
+  if (g_opt_bracket != c.bracket || g_opt_intersect != c.intersect || extra != c.extra || g_opt_cuckoo != c.cuckoo) {
+    small_set_constants(g_opt_bracket, g_opt_intersect, extra < 0 ? 0 : extra, g_opt_cuckoo);
+    large_set_constants(g_opt_bracket, g_opt_intersect, extra < 0 ? 0 : extra, g_opt_cuckoo);
+    c.cuckoo = g_opt_cuckoo;
     c.bracket = g_opt_bracket;
     c.intersect = g_opt_intersect;
     c.extra = extra;

@@ -40,6 +40,7 @@ constexpr int TS_L = TC_TS_L;         // CTA items (pieces): the table's size in
 constexpr int TS_LMAX = TC_TS_LMAX;
 constexpr uint32_t LG_SMEM_WORDS = (PIECE + 72) + ((PIECE << TS_L) + 64) / 2;  // piece (+pad) + u16 table
 constexpr uint32_t CHUNK = 8;         // worklist entries per atomic fetch
+constexpr uint32_t CK_MAXL = (PIECE * 9) / 10;  // cuckoo sets: pieces up to 0.9 x 4096 (2 x 4096 slots)
 
 struct WarpScratch {  // per-warp owner-search tables for one 32-v chunk
   uint64_t vb[32];
@@ -102,6 +103,17 @@ static __constant__ int g_bracket = 1;  // bracketed binary search on (option "b
 static __constant__ int g_merge = 0;    // sort-merge intersection instead of binary search (option "intersect")
 static __constant__ int g_extra = 0;    // MODE 3: extra searches per 8 wedges (option "extra_compute", §5.3 p_c)
 static __constant__ uint32_t g_sink_mask = 0;
+static __constant__ int g_cuckoo = 64;  // count-only CTA items: cuckoo set of the piece, max evictions per insert (0 = off)
+
+// Cuckoo hash set of a staged piece (count-only CTA items, option "cuckoo"): two tables of
+// M = 2^b slots in shared memory, w at T1[h1(w)] or T2[h2(w)] (multiplicative hashes), built
+// by the CTA with atomicExch evictions (Alcantara et al.'s GPU cuckoo insertion).  A probe is
+// two independent 32-bit shared loads, where the bracketed binary search needs one table
+// load and S2 + 1 dependent ones: the count kernel is bound by shared-memory wavefronts.
+// Load <= 0.45 of the 2M slots (pieces up to 0.9 M elements); a failed insertion falls back
+// to the staged sorted piece.
+constexpr uint32_t CK_K1 = 0x9E3779B1u, CK_K2 = 0x85EBCA77u;
+constexpr uint32_t CK_EMPTY = 0xffffffffu;  // never a vertex id
 
 // Sort-merge intersection (the strategy the paper compares binary search against, §6.2,
 // P:548-550, Fig.10): lane l intersects N+(u) (`list`, ascending, shared or global) with
@@ -205,6 +217,17 @@ struct TabSearch {
     }
     pos = sbase + ((p - sa) >> 2);
     return lds32(p) == w;
+  }
+};
+
+struct CuckooSearch {
+  uint32_t t1, t2;  // byte addresses of the two tables
+  uint32_t sh;      // 32 - b
+  __device__ __forceinline__ bool operator()(uint32_t w, uint32_t &pos) const {
+    pos = 0;  // membership only
+    const uint32_t a1 = t1 + (((w * CK_K1) >> sh) << 2);
+    const uint32_t a2 = t2 + (((w * CK_K2) >> sh) << 2);
+    return (lds32(a1) == w) | (lds32(a2) == w);
   }
 };
 
@@ -397,13 +420,13 @@ __device__ __forceinline__ int warp_table(uint32_t sbase, uint32_t tbase, uint32
 // lies in list[0..L) (w restricted to [lo, hi]).  `padded`: list is the shared-memory copy
 // tc_smem[sbase ..] padded with +inf to 2^ceil(log2 L) (+64) entries; tbase != ~0: room
 // for a bracket table.  Returns this lane's matches.
-template <int MODE, int NB = 4>
+template <int MODE, int NB = 4, bool CK = false>
 __device__ __forceinline__ uint32_t warp_chunk(const uint64_t *__restrict__ offs, const uint32_t *__restrict__ col,
                                                uint32_t v, bool valid, const uint32_t *list, uint32_t sbase,
                                                uint32_t tbase, uint32_t cbase, uint32_t L, bool padded, uint32_t lo,
                                                uint32_t hi, WarpScratch &ws, unsigned long long *tv, uint32_t vidx,
                                                uint64_t ua, uint64_t ebase, uint32_t vbits, int S2pre = -1,
-                                               uint32_t shpre = 0, int abspre = 0) {
+                                               uint32_t shpre = 0, int abspre = 0, uint32_t ck_sh = 0) {
   constexpr bool PV = MODE == 1, PE = MODE == 2;
   const unsigned lane = lane_id();
   uint64_t vb = 0;
@@ -427,7 +450,11 @@ __device__ __forceinline__ uint32_t warp_chunk(const uint64_t *__restrict__ offs
   __syncwarp();
   uint32_t cnt = 0;
   if (MODE == 0 && g_merge) return merge_lane(list, L, col + vb, dv);
-  if (total) {
+  if (CK && MODE == 0 && ck_sh && total) {  // cuckoo hash set at tc_smem[sbase ..] (2 x 2^(32-ck_sh) slots)
+    const uint32_t t1 = smem_addr(sbase);
+    cnt = wedge_loop<MODE, CuckooSearch, NB>(col, CuckooSearch{t1, t1 + (4u << (32 - ck_sh)), ck_sh}, sbase,
+                                             cbase, st_lane, total, ws, tv, ebase);
+  } else if (total) {
     const int S = padded ? ceil_log2(L) : 0;
     int S2 = S2pre >= 0 ? S2pre : 99;  // S2pre: table prebuilt by the CTA (large kernel)
     uint32_t sh = shpre;
@@ -700,6 +727,7 @@ __global__ __launch_bounds__(LG_THREADS, OWN ? TC_LG_MINB_OWN : 5) void count_la
   __shared__ __align__(8) uint64_t s_bar;
   __shared__ unsigned long long s_item;
   __shared__ uint32_t s_next;  // next sub-chunk of the current piece
+  __shared__ uint32_t s_ckfail;  // cuckoo insertion failed (fall back to the sorted piece)
   WarpScratch &ws = s_ws[warp_id()];
   if (threadIdx.x == 0) mbar_init(&s_bar, 1);
   __syncthreads();
@@ -734,11 +762,43 @@ __global__ __launch_bounds__(LG_THREADS, OWN ? TC_LG_MINB_OWN : 5) void count_la
     uint64_t ucnt = 0;
     for (uint32_t p0 = 0; p0 < L; p0 += PIECE) {
       const uint32_t plen = min(PIECE, L - p0);
+      uint32_t ck_sh = 0;  // cuckoo set of the piece (count only), 0 = sorted piece
+      if (MODE == 0 && g_cuckoo && !g_merge && plen <= CK_MAXL && cbeg < cend) {
+        const int b = max(6, ceil_log2((plen * 10 + 8) / 9));  // 2^b >= plen / 0.9
+        const uint32_t M = 1u << b;
+        for (uint32_t j = threadIdx.x; j < 2 * M; j += LG_THREADS) tc_smem[j] = CK_EMPTY;
+        if (threadIdx.x == 0) {
+          s_ckfail = 0;
+          s_next = 0;
+        }
+        __syncthreads();
+        for (uint32_t j = threadIdx.x; j < plen; j += LG_THREADS) {
+          uint32_t x = ldg_u32(col + a + p0 + j);
+          uint32_t tb = 0;
+          for (int it = 0; it < g_cuckoo && x != CK_EMPTY; ++it) {  // the evicted element moves to its other table
+            const uint32_t idx = tb ? M + ((x * CK_K2) >> (32 - b)) : ((x * CK_K1) >> (32 - b));
+            x = atomicExch(&tc_smem[idx], x);
+            tb ^= 1u;
+          }
+          if (x != CK_EMPTY) s_ckfail = 1;
+        }
+        __syncthreads();
+        if (!s_ckfail) ck_sh = 32 - b;
+        __syncthreads();  // s_ckfail read by every thread before any reset
+      }
+      uint32_t shift = 0;
+      const uint32_t *list = s_piece;
+      uint32_t lo = 0, hi = 0;
+      int S2 = -1;
+      uint32_t sh = 0;
+      bool abs_t = false;
+      uint32_t tbase = 0;
+      if (!ck_sh) {
       // 16-byte aligned bulk copy covering col[a+p0, a+p0+plen)
       const uint64_t first = a + p0;
       const uint64_t abeg = first & ~3ull;             // element index, 16 B aligned
       const uint64_t aend = (first + plen + 3) & ~3ull;
-      const uint32_t shift = (uint32_t)(first - abeg);
+      shift = (uint32_t)(first - abeg);
       if (threadIdx.x == 0) {
         unsigned bytes = (unsigned)((aend - abeg) * 4);
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // prior generic reads of the piece
@@ -748,20 +808,18 @@ __global__ __launch_bounds__(LG_THREADS, OWN ? TC_LG_MINB_OWN : 5) void count_la
       mbar_wait(&s_bar, phase);
       if (threadIdx.x == 0) s_next = 0;  // published by the barrier below
       phase ^= 1u;
-      const uint32_t *list = s_piece + shift;
+      list = s_piece + shift;
       // pad the piece with +inf up to a power of two (+64) for the fixed-depth search; the
       // bracket table starts right after it (u16 entries, 4-byte aligned)
       const uint32_t P = (1u << ceil_log2(plen)) + 64;
       for (uint32_t j = plen + threadIdx.x; j < P; j += LG_THREADS) s_piece[shift + j] = 0xffffffffu;
       __syncthreads();
-      const uint32_t tbase = shift + P;
+      tbase = shift + P;
       const uint32_t tcap = (LG_SMEM_WORDS - tbase) * 2u;  // table entries that fit
-      const uint32_t lo = list[0], hi = list[plen - 1];
+      lo = list[0];
+      hi = list[plen - 1];
       // CTA-wide bracket table of the piece (shared by all warps of the item); absolute
       // (bucket w >> sh over [0, 2^vbits)) when the piece spans the whole label range
-      int S2 = -1;
-      uint32_t sh = 0;
-      bool abs_t = false;
       const int S = ceil_log2(plen);
       if (g_bracket && S >= 6) {
         const int span_bits = 32 - __clz(hi - lo);
@@ -792,6 +850,7 @@ __global__ __launch_bounds__(LG_THREADS, OWN ? TC_LG_MINB_OWN : 5) void count_la
         if (S2 > 6) S2 = -1;  // pathological skew: plain fixed-depth search
         __syncthreads();
       }
+      }  // sorted piece
       uint32_t cnt = 0;
       // the item's v's in sub-chunks of LG_SUB fetched dynamically by the warps: the
       // wedges behind each v vary widely, and a static 32-v share per warp left warps
@@ -804,9 +863,9 @@ __global__ __launch_bounds__(LG_THREADS, OWN ? TC_LG_MINB_OWN : 5) void count_la
         if (c0 >= cend) break;
         const bool valid = lane_id() < SUB && c0 + lane_id() < cend;
         const uint32_t v = valid ? ldg_u32(olist + c0 + lane_id()) : 0u;
-        cnt += warp_chunk<MODE, MODE == 0 ? 8 : 4>(offs, col, v, valid, list, shift, S2 >= 0 ? tbase : 0xffffffffu, 0xffffffffu, plen,
+        cnt += warp_chunk<MODE, MODE == 0 ? 8 : 4, true>(offs, col, v, valid, list, shift, S2 >= 0 ? tbase : 0xffffffffu, 0xffffffffu, plen,
                                 true, lo, hi, ws, tv, c0 + lane_id(), a, a + p0, vbits, S2 >= 0 ? S2 : -2, sh,
-                                abs_t ? 1 : 0);
+                                abs_t ? 1 : 0, ck_sh);
       }
       ucnt += cnt;
       __syncthreads();  // piece fully consumed before the next bulk copy overwrites it
@@ -865,8 +924,8 @@ const void *small_kernel(int mode, bool own);
 const void *range_kernel(int mode);
 const void *large_kernel(int mode, bool own);
 // the __constant__ options of each kernel translation unit (current device)
-void small_set_constants(int bracket, int merge, int extra);
-void large_set_constants(int bracket, int merge, int extra);
+void small_set_constants(int bracket, int merge, int extra, int cuckoo);
+void large_set_constants(int bracket, int merge, int extra, int cuckoo);
 
 }  // namespace cnt
 }  // namespace tc

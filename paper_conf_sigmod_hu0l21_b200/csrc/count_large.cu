@@ -16,7 +16,8 @@ const void *large_kernel(int mode, bool own) {
   }
 }
 
-void large_set_constants(int bracket, int merge, int extra) {
+void large_set_constants(int bracket, int merge, int extra, int cuckoo) {
+  TC_CUDA(cudaMemcpyToSymbol(g_cuckoo, &cuckoo, sizeof(int)));
   TC_CUDA(cudaMemcpyToSymbol(g_bracket, &bracket, sizeof(int)));
   TC_CUDA(cudaMemcpyToSymbol(g_merge, &merge, sizeof(int)));
   TC_CUDA(cudaMemcpyToSymbol(g_extra, &extra, sizeof(int)));

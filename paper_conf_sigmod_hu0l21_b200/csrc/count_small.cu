@@ -26,7 +26,8 @@ const void *range_kernel(int mode) {
   }
 }
 
-void small_set_constants(int bracket, int merge, int extra) {
+void small_set_constants(int bracket, int merge, int extra, int cuckoo) {
+  TC_CUDA(cudaMemcpyToSymbol(g_cuckoo, &cuckoo, sizeof(int)));
   TC_CUDA(cudaMemcpyToSymbol(g_bracket, &bracket, sizeof(int)));
   TC_CUDA(cudaMemcpyToSymbol(g_merge, &merge, sizeof(int)));
   TC_CUDA(cudaMemcpyToSymbol(g_extra, &extra, sizeof(int)));

@@ -516,6 +516,30 @@ def test_owner_tiles(cap):
         tc.tc_set_option("small_cap", 256)
 
 
+@pytest.mark.parametrize("evictions", [0, 1, 2, 64])
+def test_cuckoo_piece_sets(evictions):
+    """Count-only CTA items with the staged list as a cuckoo set (option cuckoo = eviction
+    limit): off (0), mostly failing inserts that fall back to the sorted piece (1, 2) and the
+    default (64) all give the oracle's T, on both the owner and the classic schedule, with
+    single- and multi-piece lists."""
+    tc.tc_set_option("cuckoo", evictions)
+    tc.tc_set_option("small_cap", 32)
+    try:
+        for seed, (sc, ef, d, r) in enumerate(((13, 32, "degree", "paper"), (12, 16, "id", "none"))):
+            spec = graphgen.rmat_spec(sc, ef, 970 + seed)
+            src, dst = graphgen.generate_cpu(spec)
+            ref = oracle.run(src, dst, spec.n, d, r)
+            g = tc.Graph(src, dst, spec.n).direct(d).reorder(r)
+            for shorter in (1, 0):
+                tc.tc_set_option("shorter", shorter)
+                assert g.count() == ref["T"], (seed, evictions, shorter)
+            g.free()
+    finally:
+        tc.tc_set_option("cuckoo", 64)
+        tc.tc_set_option("shorter", 1)
+        tc.tc_set_option("small_cap", 256)
+
+
 def test_extra_compute_instrumented_kernel_counts_unchanged():
     """The §5.3 balance-point instrumentation (option extra_compute, MODE 3: p_c extra
     searches per wedge, results discarded) leaves T and t(v) equal to the oracle's."""
