@@ -413,18 +413,22 @@ static void aorder_core(size_t n, SF S, AF active, uint32_t k, int order, uint32
     // loop over that bin (a grown key lands in a later bin whenever the bin is narrower
     // than the smallest increment); a key re-entering the current bin goes through the
     // queue's small heap and the step-by-step path.  full(pk) records a bucket that left.
-    auto phase = [&](size_t nu, auto inc, uint32_t *brec, uint32_t *rrec, auto full) {
+    // fill counts as bytes when k < 256 (the bucket counters stay cache-resident)
+    std::vector<uint8_t> fill8(k < 256 ? b : 0, 0);
+    auto phase = [&](size_t nu, auto inc, uint32_t *brec, uint32_t *rrec, auto full, auto *fl) {
       size_t i = 0;
       while (i < nu) {
         if (q.heap.empty() && q.rpos < q.run.size()) {
           const uint64_t *rp = q.run.data();
-          const size_t jend = std::min(q.run.size(), q.rpos + (nu - i));
+          const size_t rsz = q.run.size();
+          const size_t jend = std::min(rsz, q.rpos + (nu - i));
           size_t j = q.rpos;
           bool reentered = false;
           for (; j < jend; ++j, ++i) {
+            if (j + 16 < rsz) __builtin_prefetch(&fl[rp[j + 16] & imask], 1);
             const uint64_t pk = rp[j];
             const size_t bk = (size_t)(pk & imask);
-            const uint32_t r = fill[bk]++;
+            const uint32_t r = fl[bk]++;
             brec[i] = (uint32_t)bk;
             rrec[i] = r;
             const uint64_t npk = pk + inc(i);
@@ -448,7 +452,7 @@ static void aorder_core(size_t n, SF S, AF active, uint32_t k, int order, uint32
         }
         const uint64_t pk = q.top();
         const size_t bk = (size_t)(pk & imask);
-        const uint32_t r = fill[bk]++;
+        const uint32_t r = fl[bk]++;
         brec[i] = (uint32_t)bk;
         rrec[i] = r;
         const uint64_t npk = pk + inc(i);
@@ -461,9 +465,15 @@ static void aorder_core(size_t n, SF S, AF active, uint32_t k, int order, uint32
     for (size_t i = 0; i < b; ++i) keys.push_back(pack(i, 0, false));
     q.build(keys, max_pk, smin1 == INT64_MAX ? 0 : (uint64_t)smin1 << ib, ib);  // line 2: min queue
     // lines 5-9: memory-dominated v -> min bucket (line 6-7), mem_sup += S(v) (line 8), re-queue (line 9)
-    phase(
+    auto run_phase = [&](size_t nu, auto inc, uint32_t *brec, uint32_t *rrec, auto full) {
+      if (k < 256) phase(nu, inc, brec, rrec, full, fill8.data());
+      else phase(nu, inc, brec, rrec, full, fill.data());
+    };
+    run_phase(
         nmem, [&](size_t i) { return (uint64_t)smem[i] << ib; }, bmem, rmem,
         [&](size_t bk, uint64_t npk) { mem_sup[bk] = (int64_t)(npk >> ib) - off; });
+    if (k < 256)
+      for (size_t i = 0; i < b; ++i) fill[i] = fill8[i];
     q.for_each([&](uint64_t pk) { mem_sup[pk & imask] = (int64_t)(pk >> ib) - off; });
     if (trace_on()) t2 = now_ms();
     keys.clear();
@@ -471,9 +481,11 @@ static void aorder_core(size_t n, SF S, AF active, uint32_t k, int order, uint32
       if (fill[i] < k) keys.push_back(pack(i, mem_sup[i], true));
     q.build(keys, max_pk, smin2 == INT64_MAX ? 0 : (uint64_t)smin2 << ib, ib);  // line 10: max queue
     // lines 11-15: computing-dominated v -> max bucket, mem_sup += S(v) <= 0 (its negated key grows)
-    phase(
+    run_phase(
         ncomp, [&](size_t i) { return (uint64_t)(-scomp[i]) << ib; }, bcomp, rcomp,
         [&](size_t bk, uint64_t npk) { mem_sup[bk] = off - (int64_t)(npk >> ib); });
+    if (k < 256)
+      for (size_t i = 0; i < b; ++i) fill[i] = fill8[i];
     q.for_each([&](uint64_t pk) { mem_sup[pk & imask] = off - (int64_t)(pk >> ib); });
   } else if (b) {
     // generic tournament tree (mem_sup beyond the packed range)

@@ -338,16 +338,33 @@ __device__ __forceinline__ void fast_block(const uint32_t *__restrict__ p, const
 // owner of each block's first wedge is tracked warp-uniformly; a block that lies entirely
 // in that owner's list (long N+(v): most wedges of a skewed graph) takes fast_block, the
 // others walk per lane from there (wedge_block).
-template <int MODE, class Search, int NB = 4>
+// L2 prefetch (PF > 0, CTA items): the lists PF owners ahead of the one being gathered are
+// requested into L2 (one 128-B line per lane).  Measured slower on B200 (configs[3] count
+// 283 / 298 / 301 / 310 ms at PF = 0 / 1 / 2 / 4): off (TC_PF = 0, compiled out).
+#ifndef TC_PF
+#define TC_PF 0
+#endif
+template <int MODE, class Search, int NB = 4, int PF = 0>
 __device__ __forceinline__ uint32_t wedge_loop(const uint32_t *__restrict__ col, const Search &search, uint32_t sbase,
                                                uint32_t cbase, uint32_t st_lane, uint32_t total,
-                                               WarpScratch &ws, unsigned long long *tv, uint64_t ebase) {
+                                               WarpScratch &ws, unsigned long long *tv, uint64_t ebase,
+                                               uint32_t nown = 0) {
   constexpr bool FAST = MODE == 0 || MODE == 3 || MODE == 4;
   uint32_t cnt = 0;
   uint32_t uo = 0, uo_end = ws.pre[0];
   const uint32_t *uob = col + ws.vb[0];  // element j of the uniform owner's list is uob[j]
   const uint32_t last = total - 1, steps = (total + 31) >> 5, lane = lane_id();
   (void)st_lane;  // (a warp-reduction owner lookup for short lists was measured slower)
+  auto pf_list = [&](uint32_t o) {  // warp-uniform o
+    if (o >= nown) return;
+    const uint32_t b0 = o ? ws.pre[o - 1] : 0u;
+    const uintptr_t p0 = (uintptr_t)(col + ws.vb[o]);
+    const uintptr_t p1 = p0 + 4ull * (ws.pre[o] - b0);
+    for (uintptr_t q = (p0 & ~(uintptr_t)127) + 128ull * lane; q < p1; q += 4096)
+      asm volatile("prefetch.global.L2 [%0];" ::"l"(q));
+  };
+  if (PF)
+    for (uint32_t d = 1; d <= (uint32_t)PF; ++d) pf_list(d);
   auto block = [&](auto nconst, uint32_t st) {
     constexpr int N = decltype(nconst)::value;
     const uint32_t base = 32 * st;
@@ -356,6 +373,7 @@ __device__ __forceinline__ uint32_t wedge_loop(const uint32_t *__restrict__ col,
       ++uo;
       uo_end = ws.pre[uo];
       uob = col + ws.vb[uo] - b0;
+      if (PF) pf_list(uo + PF);
     }
     if (FAST && uo_end >= base + 32 * N) {
       fast_block<N, MODE>(uob + base + lane, search, base + lane, cnt);
@@ -452,8 +470,8 @@ __device__ __forceinline__ uint32_t warp_chunk(const uint64_t *__restrict__ offs
   if (MODE == 0 && g_merge) return merge_lane(list, L, col + vb, dv);
   if (CK && MODE == 0 && ck_sh && total) {  // cuckoo hash set at tc_smem[sbase ..] (2 x 2^(32-ck_sh) slots)
     const uint32_t t1 = smem_addr(sbase);
-    cnt = wedge_loop<MODE, CuckooSearch, NB>(col, CuckooSearch{t1, t1 + (4u << (32 - ck_sh)), ck_sh}, sbase,
-                                             cbase, st_lane, total, ws, tv, ebase);
+    cnt = wedge_loop<MODE, CuckooSearch, NB, TC_PF>(col, CuckooSearch{t1, t1 + (4u << (32 - ck_sh)), ck_sh}, sbase,
+                                                    cbase, st_lane, total, ws, tv, ebase, (uint32_t)__popc(nz));
   } else if (total) {
     const int S = padded ? ceil_log2(L) : 0;
     int S2 = S2pre >= 0 ? S2pre : 99;  // S2pre: table prebuilt by the CTA (large kernel)
