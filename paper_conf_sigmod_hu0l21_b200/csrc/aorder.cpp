@@ -17,11 +17,13 @@
 //   F_m = BW(d)^α (Eq.19), F_c = 1/d^β (Eq.20); α = β = 1/2 evaluated literally as
 //   sqrt(BW(d)) and sqrt(1/d) (Eq.22); BW(d) = d unless a table is given (Q15).
 #include <algorithm>
+#include <atomic>
 #include <chrono>
 #include <cstdio>
 #include <cstdlib>
 #include <cmath>
 #include <cstdint>
+#include <memory>
 #include <mutex>
 #include <stdexcept>
 #include <thread>
@@ -115,6 +117,85 @@ struct PackedTournament4 {
   }
 };
 
+// Sorts a bin's packed keys by (value, bucket index): LSD radix on the value bits below the
+// bin boundary only ([lo_bits, shift): the bin fixes the bits above, the low lo_bits are the
+// bucket index), stable; then every run of equal values is put in index order (rare, except
+// for the initial all-zero bin, which is already in index order).
+static void sort_keys(std::vector<uint64_t> &v, std::vector<uint64_t> &tmp, int lo_bits, int shift) {
+  const size_t n = v.size();
+  if (n < 64) {
+    std::sort(v.begin(), v.end());
+    return;
+  }
+  tmp.resize(n);
+  uint32_t cnt[256];
+  for (int b = lo_bits; b < shift; b += 8) {
+    const int w = std::min(8, shift - b);
+    const uint64_t mask = (1ull << w) - 1;
+    std::fill(cnt, cnt + 256, 0u);
+    for (size_t i = 0; i < n; ++i) ++cnt[(v[i] >> b) & mask];
+    uint32_t acc = 0;
+    for (uint64_t d = 0; d <= mask; ++d) {
+      const uint32_t c = cnt[d];
+      cnt[d] = acc;
+      acc += c;
+    }
+    for (size_t i = 0; i < n; ++i) tmp[cnt[(v[i] >> b) & mask]++] = v[i];
+    v.swap(tmp);
+  }
+  for (size_t i = 0; i < n;) {
+    size_t j = i + 1;
+    while (j < n && (v[j] >> lo_bits) == (v[i] >> lo_bits)) ++j;
+    if (j - i > 1 && !std::is_sorted(v.begin() + i, v.begin() + j)) std::sort(v.begin() + i, v.begin() + j);
+    i = j;
+  }
+}
+
+// Helper thread that sorts a copy of the NEXT bin while the greedy consumes the current
+// one (the bin sorts are ~30% of the sequential greedy).  Keys pushed into that bin after the
+// copy was taken (its tail) are sorted and merged in when the bin becomes current, so the
+// consumed order is exactly the single-threaded one.
+struct PreSorter {
+  std::thread th;
+  std::atomic<uint64_t> req{0}, done{0};
+  std::atomic<bool> stop{false};
+  std::vector<uint64_t> keys, tmp;  // the copy, sorted in place by the helper
+  int lo_bits = 0, shift = 0;
+  size_t bin = SIZE_MAX;            // bin of the submitted copy
+  PreSorter() {
+    th = std::thread([this] {
+      uint64_t seen = 0;
+      for (;;) {
+        uint64_t r;
+        unsigned spins = 0;
+        while ((r = req.load(std::memory_order_acquire)) == seen) {
+          if (stop.load(std::memory_order_acquire)) return;
+          if (++spins > 4096) std::this_thread::yield();
+        }
+        seen = r;
+        sort_keys(keys, tmp, lo_bits, shift);
+        done.store(r, std::memory_order_release);
+      }
+    });
+  }
+  ~PreSorter() {
+    stop.store(true, std::memory_order_release);
+    th.join();
+  }
+  void submit(size_t b, const std::vector<uint64_t> &src, int lo, int sh) {
+    keys.assign(src.begin(), src.end());
+    lo_bits = lo;
+    shift = sh;
+    bin = b;
+    req.fetch_add(1, std::memory_order_acq_rel);
+  }
+  void wait() const {
+    const uint64_t r = req.load(std::memory_order_relaxed);
+    while (done.load(std::memory_order_acquire) != r) {
+    }
+  }
+};
+
 // Monotone bucketed priority queue on the same packed keys.  In both phases only the
 // top bucket changes and its packed key only grows (phase 1 adds S > 0 to the min; phase
 // 2 adds S <= 0 to the max, i.e. its negated key grows), so the extracted minimum never
@@ -133,6 +214,7 @@ struct MonoQueue {
   size_t rpos = 0;
   std::vector<uint64_t> heap;
   size_t cur = 0;
+  double *trace_ns = nullptr;  // TC_AORDER_TRACE: time spent sorting bins
   size_t bin_of(uint64_t pk) const { return (size_t)((pk >> shift) - bin0); }
   static constexpr size_t D = 4;  // 4-ary min-heap, children 4i+1 .. 4i+4
   void sift_down(size_t i) {
@@ -170,42 +252,38 @@ struct MonoQueue {
   // ([lo_bits, shift): the bin fixes the bits above, the low lo_bits are the bucket index),
   // stable; then every run of equal values is put in index order (rare, except for the
   // initial all-zero bin, which is already in index order)
-  void sort_run() {
-    const size_t n = run.size();
-    if (n < 64) {
-      std::sort(run.begin(), run.end());
-      return;
+  void sort_run() { sort_keys(run, tmp, lo_bits, shift); }
+  PreSorter *ps = nullptr;  // optional helper thread (large queues)
+  std::vector<uint64_t> tail;
+  void activate() {  // bin `cur` becomes the sorted run
+    if (ps && ps->bin == cur) {
+      ps->wait();
+      std::vector<uint64_t> &B = bins[cur];
+      const size_t P = ps->keys.size();
+      tail.assign(B.begin() + P, B.end());
+      sort_keys(tail, tmp, lo_bits, shift);
+      run.resize(P + tail.size());
+      std::merge(ps->keys.begin(), ps->keys.end(), tail.begin(), tail.end(), run.begin());
+      B.clear();
+      ps->bin = SIZE_MAX;
+    } else {
+      run.clear();
+      run.swap(bins[cur]);
+      sort_run();
     }
-    tmp.resize(n);
-    uint32_t cnt[256];
-    for (int b = lo_bits; b < shift; b += 8) {
-      const int w = std::min(8, shift - b);
-      const uint64_t mask = (1ull << w) - 1;
-      std::fill(cnt, cnt + 256, 0u);
-      for (size_t i = 0; i < n; ++i) ++cnt[(run[i] >> b) & mask];
-      uint32_t acc = 0;
-      for (uint64_t d = 0; d <= mask; ++d) {
-        const uint32_t c = cnt[d];
-        cnt[d] = acc;
-        acc += c;
-      }
-      for (size_t i = 0; i < n; ++i) tmp[cnt[(run[i] >> b) & mask]++] = run[i];
-      run.swap(tmp);
-    }
-    for (size_t i = 0; i < n;) {
-      size_t j = i + 1;
-      while (j < n && (run[j] >> lo_bits) == (run[i] >> lo_bits)) ++j;
-      if (j - i > 1 && !std::is_sorted(run.begin() + i, run.begin() + j)) std::sort(run.begin() + i, run.begin() + j);
-      i = j;
-    }
+    rpos = 0;
+    if (ps && cur + 1 < bins.size() && bins[cur + 1].size() >= 256) ps->submit(cur + 1, bins[cur + 1], lo_bits, shift);
   }
   void refill() {
     while (rpos == run.size() && heap.empty() && cur + 1 < bins.size()) {
       ++cur;
-      run.clear();
-      run.swap(bins[cur]);
-      sort_run();
-      rpos = 0;
+      if (trace_ns) {
+        const auto t0 = std::chrono::steady_clock::now();
+        activate();
+        *trace_ns += std::chrono::duration<double, std::nano>(std::chrono::steady_clock::now() - t0).count();
+      } else {
+        activate();
+      }
     }
   }
   // keys: packed keys of the alive buckets; max_pk: upper bound of any key ever inserted;
@@ -223,10 +301,11 @@ struct MonoQueue {
     for (uint64_t k : keys) bins[bin_of(k)].push_back(k);
     cur = 0;
     heap.clear();
-    run.clear();
-    run.swap(bins[0]);
-    sort_run();
-    rpos = 0;
+    if (ps) {
+      ps->wait();
+      ps->bin = SIZE_MAX;
+    }
+    activate();
     refill();
   }
   bool empty() const { return rpos == run.size() && heap.empty(); }
@@ -315,7 +394,7 @@ static void aorder_core(size_t n, SF S, AF active, uint32_t k, int order, uint32
   AOrderWorkspace &W = workspace();
   std::lock_guard<std::mutex> lock(W.mu);
   const double t0 = trace_on() ? now_ms() : 0;
-  double t1 = 0, t2 = 0, t3 = 0;
+  double t1 = 0, t2 = 0, t3 = 0, sort_ns = 0;
   // line 3-4: V_mem / V_comp in ascending unit index: per-chunk counts (with max |S| and
   // the least nonzero |S| of each class, for the queue's key packing), then placement of
   // each unit and its S, all on the host cores
@@ -405,6 +484,13 @@ static void aorder_core(size_t n, SF S, AF active, uint32_t k, int order, uint32
       return ((uint64_t)((want_max ? -sup : sup) + off) << ib) | (uint64_t)i;
     };
     MonoQueue q;
+    if (trace_on()) q.trace_ns = &sort_ns;
+    // bin pre-sorting on a helper thread for large queues (identical output)
+    std::unique_ptr<PreSorter> presorter;
+    if (b >= 4096 && std::thread::hardware_concurrency() >= 2 && !std::getenv("TC_AORDER_NOPRESORT")) {
+      presorter.reset(new PreSorter());
+      q.ps = presorter.get();
+    }
     std::vector<uint64_t> keys;
     keys.reserve(b);
     // One phase of the greedy: unit i takes the bucket at the top of the queue and the
@@ -534,8 +620,8 @@ static void aorder_core(size_t n, SF S, AF active, uint32_t k, int order, uint32
       if (!active(v)) perm[v] = idx++;
   });
   if (trace_on())
-    fprintf(stderr, "aorder n=%zu mem=%zu comp=%zu b=%zu: classify %.1f ms, phase1 %.1f, phase2 %.1f, relabel %.1f\n",
-            n, nmem, ncomp, b, t1 - t0, t2 - t1, t3 - t2, now_ms() - t3);
+    fprintf(stderr, "aorder n=%zu mem=%zu comp=%zu b=%zu: classify %.1f ms, phase1 %.1f, phase2 %.1f (bin sorts %.1f), relabel %.1f\n",
+            n, nmem, ncomp, b, t1 - t0, t2 - t1, t3 - t2, sort_ns / 1e6, now_ms() - t3);
 }
 
 
