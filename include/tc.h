@@ -239,7 +239,10 @@ tc_status tc_export_units(tc_graph *g, uint64_t *units, uint32_t *unit_off);
  * items: the staged list is held as a cuckoo hash set — two tables of 2^b slots, probe =
  * two independent shared loads — instead of the sorted piece with its bracket table; the
  * value is the eviction limit per insertion, default 64, 0 = off; an insertion that fails
- * falls back to the sorted piece, counts are unchanged). */
+ * falls back to the sorted piece, counts are unchanged), "aorder_device" (1 = default: the
+ * A-order classification into memory- / computing-dominated vertices (Alg.2 lines 3-4) and
+ * the relabel (lines 16-20) run on the device around the host's sequential greedy; 0 = all
+ * on the host; identical pi). */
 tc_status tc_set_option(const char *key, int64_t value);
 
 /* Per-kernel profile since the last reset, as JSON text into buf (host, cap bytes):

@@ -388,88 +388,21 @@ static double now_ms() {
   return std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now().time_since_epoch()).count();
 }
 
-template <class SF, class AF>
-static void aorder_core(size_t n, SF S, AF active, uint32_t k, int order, uint32_t *perm,
-                        std::vector<uint32_t> &bucket_off, int64_t &eq3) {
-  AOrderWorkspace &W = workspace();
-  std::lock_guard<std::mutex> lock(W.mu);
-  const double t0 = trace_on() ? now_ms() : 0;
-  double t1 = 0, t2 = 0, t3 = 0, sort_ns = 0;
-  // line 3-4: V_mem / V_comp in ascending unit index: per-chunk counts (with max |S| and
-  // the least nonzero |S| of each class, for the queue's key packing), then placement of
-  // each unit and its S, all on the host cores
-  const unsigned T = host_threads(n);
-  std::vector<size_t> cm(T + 1, 0), cc(T + 1, 0), ci(T + 1, 0);
-  std::vector<int64_t> tmax(T, 0), tmin1(T, INT64_MAX), tmin2(T, INT64_MAX);
-  par_chunks(n, T, [&](size_t lo, size_t hi, unsigned t) {
-    size_t a = 0, c = 0, z = 0;
-    int64_t mx = 0, m1 = INT64_MAX, m2 = INT64_MAX;
-    for (size_t v = lo; v < hi; ++v) {
-      if (!active(v)) {
-        ++z;
-        continue;
-      }
-      const int64_t sv = S(v), av = std::llabs(sv);
-      mx = std::max(mx, av);
-      if (sv > 0) {
-        ++a;
-        m1 = std::min(m1, av);
-      } else {
-        ++c;
-        if (av) m2 = std::min(m2, av);
-      }
-    }
-    cm[t + 1] = a;
-    cc[t + 1] = c;
-    ci[t + 1] = z;
-    tmax[t] = mx;
-    tmin1[t] = m1;
-    tmin2[t] = m2;
-  });
-  int64_t smax = 0, smin1 = INT64_MAX, smin2 = INT64_MAX;  // max |S|; min nonzero |S| per phase
-  for (unsigned t = 0; t < T; ++t) {
-    cm[t + 1] += cm[t];
-    cc[t + 1] += cc[t];
-    ci[t + 1] += ci[t];
-    smax = std::max(smax, tmax[t]);
-    smin1 = std::min(smin1, tmin1[t]);
-    smin2 = std::min(smin2, tmin2[t]);
-  }
-  const size_t nmem = cm[T], ncomp = cc[T];
-  uint32_t *vmem = grow(W.vmem, nmem), *vcomp = grow(W.vcomp, ncomp);
-  int64_t *smem = grow(W.smem, nmem), *scomp = grow(W.scomp, ncomp);
-  par_chunks(n, T, [&](size_t lo, size_t hi, unsigned t) {
-    size_t a = cm[t], c = cc[t];
-    for (size_t v = lo; v < hi; ++v) {
-      if (!active(v)) continue;
-      const int64_t sv = S(v);
-      if (sv > 0) {
-        smem[a] = sv;
-        vmem[a++] = (uint32_t)v;
-      } else {
-        scomp[c] = sv;
-        vcomp[c++] = (uint32_t)v;
-      }
-    }
-  });
-  if (order == 1) {  // LPT option (Q18): descending |S|, ties by index
-    auto lpt = [&](uint32_t a, uint32_t b) {
-      int64_t x = std::llabs(S(a)), y = std::llabs(S(b));
-      return x != y ? x > y : a < b;
-    };
-    std::sort(vmem, vmem + nmem, lpt);
-    std::sort(vcomp, vcomp + ncomp, lpt);
-    for (size_t i = 0; i < nmem; ++i) smem[i] = S(vmem[i]);
-    for (size_t i = 0; i < ncomp; ++i) scomp[i] = S(vcomp[i]);
-  }
-  if (trace_on()) t1 = now_ms();
+// Lines 1-20 of Algorithm 2 after the classification (lines 3-4): memory-dominated units
+// (superiority SMEM(i) > 0, i < nmem, in placement order) then computing-dominated ones
+// (SCOMP(i) <= 0); records bucket / rank per placement, bucket_off (buckets in index order,
+// members in insertion order) and the Eq.3 objective.  smax = max |S|, smin1 = least S > 0,
+// smin2 = least nonzero |S| of the computing-dominated units (INT64_MAX when none).
+template <class SMF, class SCF>
+static void aorder_greedy(size_t nmem, SMF SMEM, size_t ncomp, SCF SCOMP, int64_t smax, int64_t smin1, int64_t smin2,
+                          uint32_t k, uint32_t *bmem, uint32_t *rmem, uint32_t *bcomp, uint32_t *rcomp,
+                          std::vector<uint32_t> &bucket_off, int64_t &eq3, double *tr) {
+  double t2 = 0, sort_ns = 0;
   const size_t nact = nmem + ncomp;
   const size_t b = (nact + k - 1) / k;
   std::vector<int64_t> mem_sup(b, 0);        // line 1
   std::vector<uint32_t> fill(b, 0);
   // insertion record per placement index (sequential writes; the relabel scatters them)
-  uint32_t *bmem = grow(W.bmem, nmem), *rmem = grow(W.rmem, nmem);
-  uint32_t *bcomp = grow(W.bcomp, ncomp), *rcomp = grow(W.rcomp, ncomp);
   const int ib = b > 1 ? 64 - __builtin_clzll((unsigned long long)(b - 1)) : 1;
   const long double bound = (long double)smax * (long double)k * 2.0L + 2.0L;  // |mem_sup| < k smax
   const bool packed = bound * (long double)(1ull << ib) < 9.0e18L;
@@ -556,7 +489,7 @@ static void aorder_core(size_t n, SF S, AF active, uint32_t k, int order, uint32
       else phase(nu, inc, brec, rrec, full, fill.data());
     };
     run_phase(
-        nmem, [&](size_t i) { return (uint64_t)smem[i] << ib; }, bmem, rmem,
+        nmem, [&](size_t i) { return (uint64_t)SMEM(i) << ib; }, bmem, rmem,
         [&](size_t bk, uint64_t npk) { mem_sup[bk] = (int64_t)(npk >> ib) - off; });
     if (k < 256)
       for (size_t i = 0; i < b; ++i) fill[i] = fill8[i];
@@ -568,7 +501,7 @@ static void aorder_core(size_t n, SF S, AF active, uint32_t k, int order, uint32
     q.build(keys, max_pk, smin2 == INT64_MAX ? 0 : (uint64_t)smin2 << ib, ib);  // line 10: max queue
     // lines 11-15: computing-dominated v -> max bucket, mem_sup += S(v) <= 0 (its negated key grows)
     run_phase(
-        ncomp, [&](size_t i) { return (uint64_t)(-scomp[i]) << ib; }, bcomp, rcomp,
+        ncomp, [&](size_t i) { return (uint64_t)(-SCOMP(i)) << ib; }, bcomp, rcomp,
         [&](size_t bk, uint64_t npk) { mem_sup[bk] = off - (int64_t)(npk >> ib); });
     if (k < 256)
       for (size_t i = 0; i < b; ++i) fill[i] = fill8[i];
@@ -583,7 +516,7 @@ static void aorder_core(size_t n, SF S, AF active, uint32_t k, int order, uint32
       const int64_t bk = q.top();                // line 6
       bmem[i] = (uint32_t)bk;                    // line 7
       rmem[i] = fill[bk]++;
-      mem_sup[bk] += smem[i];                    // line 8
+      mem_sup[bk] += SMEM(i);                    // line 8
       if (fill[bk] == k) alive[bk] = 0;
       q.update((size_t)bk, mem_sup[bk], alive[bk]);  // line 9
     }
@@ -593,20 +526,110 @@ static void aorder_core(size_t n, SF S, AF active, uint32_t k, int order, uint32
       const int64_t bk = q.top();                // line 12
       bcomp[i] = (uint32_t)bk;                   // line 13
       rcomp[i] = fill[bk]++;
-      mem_sup[bk] += scomp[i];                   // line 14
+      mem_sup[bk] += SCOMP(i);                   // line 14
       if (fill[bk] == k) alive[bk] = 0;
       q.update((size_t)bk, mem_sup[bk], alive[bk]);  // line 15
     }
   }
-  if (trace_on()) t3 = now_ms();
-  // line 16-20: buckets in index order, members in insertion order (bucket start + rank);
-  // inactive units last in unit order (Q16)
+  if (tr) {
+    tr[0] = t2;
+    tr[1] = sort_ns;
+  }
+  // line 16-20: bucket offsets; Eq.3 objective (λ folded into S)
   bucket_off.assign(b + 1, 0);
   eq3 = 0;
   for (size_t i = 0; i < b; ++i) {
     bucket_off[i + 1] = bucket_off[i] + fill[i];
-    eq3 += std::llabs(mem_sup[i]);           // Eq.3 objective (λ folded into S)
+    eq3 += std::llabs(mem_sup[i]);
   }
+}
+
+template <class SF, class AF>
+static void aorder_core(size_t n, SF S, AF active, uint32_t k, int order, uint32_t *perm,
+                        std::vector<uint32_t> &bucket_off, int64_t &eq3) {
+  AOrderWorkspace &W = workspace();
+  std::lock_guard<std::mutex> lock(W.mu);
+  const double t0 = trace_on() ? now_ms() : 0;
+  double t1 = 0, t3 = 0;
+  // line 3-4: V_mem / V_comp in ascending unit index: per-chunk counts (with max |S| and
+  // the least nonzero |S| of each class, for the queue's key packing), then placement of
+  // each unit and its S, all on the host cores
+  const unsigned T = host_threads(n);
+  std::vector<size_t> cm(T + 1, 0), cc(T + 1, 0), ci(T + 1, 0);
+  std::vector<int64_t> tmax(T, 0), tmin1(T, INT64_MAX), tmin2(T, INT64_MAX);
+  par_chunks(n, T, [&](size_t lo, size_t hi, unsigned t) {
+    size_t a = 0, c = 0, z = 0;
+    int64_t mx = 0, m1 = INT64_MAX, m2 = INT64_MAX;
+    for (size_t v = lo; v < hi; ++v) {
+      if (!active(v)) {
+        ++z;
+        continue;
+      }
+      const int64_t sv = S(v), av = std::llabs(sv);
+      mx = std::max(mx, av);
+      if (sv > 0) {
+        ++a;
+        m1 = std::min(m1, av);
+      } else {
+        ++c;
+        if (av) m2 = std::min(m2, av);
+      }
+    }
+    cm[t + 1] = a;
+    cc[t + 1] = c;
+    ci[t + 1] = z;
+    tmax[t] = mx;
+    tmin1[t] = m1;
+    tmin2[t] = m2;
+  });
+  int64_t smax = 0, smin1 = INT64_MAX, smin2 = INT64_MAX;  // max |S|; min nonzero |S| per phase
+  for (unsigned t = 0; t < T; ++t) {
+    cm[t + 1] += cm[t];
+    cc[t + 1] += cc[t];
+    ci[t + 1] += ci[t];
+    smax = std::max(smax, tmax[t]);
+    smin1 = std::min(smin1, tmin1[t]);
+    smin2 = std::min(smin2, tmin2[t]);
+  }
+  const size_t nmem = cm[T], ncomp = cc[T];
+  uint32_t *vmem = grow(W.vmem, nmem), *vcomp = grow(W.vcomp, ncomp);
+  int64_t *smem = grow(W.smem, nmem), *scomp = grow(W.scomp, ncomp);
+  par_chunks(n, T, [&](size_t lo, size_t hi, unsigned t) {
+    size_t a = cm[t], c = cc[t];
+    for (size_t v = lo; v < hi; ++v) {
+      if (!active(v)) continue;
+      const int64_t sv = S(v);
+      if (sv > 0) {
+        smem[a] = sv;
+        vmem[a++] = (uint32_t)v;
+      } else {
+        scomp[c] = sv;
+        vcomp[c++] = (uint32_t)v;
+      }
+    }
+  });
+  if (order == 1) {  // LPT option (Q18): descending |S|, ties by index
+    auto lpt = [&](uint32_t a, uint32_t b) {
+      int64_t x = std::llabs(S(a)), y = std::llabs(S(b));
+      return x != y ? x > y : a < b;
+    };
+    std::sort(vmem, vmem + nmem, lpt);
+    std::sort(vcomp, vcomp + ncomp, lpt);
+    for (size_t i = 0; i < nmem; ++i) smem[i] = S(vmem[i]);
+    for (size_t i = 0; i < ncomp; ++i) scomp[i] = S(vcomp[i]);
+  }
+  if (trace_on()) t1 = now_ms();
+  uint32_t *bmem = grow(W.bmem, nmem), *rmem = grow(W.rmem, nmem);
+  uint32_t *bcomp = grow(W.bcomp, ncomp), *rcomp = grow(W.rcomp, ncomp);
+  double tr[2] = {0, 0};
+  aorder_greedy(
+      nmem, [&](size_t i) { return smem[i]; }, ncomp, [&](size_t i) { return scomp[i]; }, smax, smin1, smin2, k, bmem,
+      rmem, bcomp, rcomp, bucket_off, eq3, trace_on() ? tr : nullptr);
+  const double t2 = tr[0], sort_ns = tr[1];
+  const size_t b = bucket_off.size() - 1;
+  if (trace_on()) t3 = now_ms();
+  // line 16-20: buckets in index order, members in insertion order (bucket start + rank);
+  // inactive units last in unit order (Q16)
   const uint32_t inactive0 = bucket_off[b];
   par_chunks(nmem, T, [&](size_t lo, size_t hi, unsigned) {
     for (size_t i = lo; i < hi; ++i) perm[vmem[i]] = bucket_off[bmem[i]] + rmem[i];
@@ -649,6 +672,27 @@ void aorder_host(const uint32_t *od, size_t n, const tc_aorder_params &p, uint32
   aorder_core(
       n, [&](size_t v) -> int64_t { return use_table ? table[od[v]] : memory_superiority(od[v], p); },
       [&](size_t v) { return od[v] != 0; }, p.k, p.order, perm, bucket_off, eq3);
+}
+
+// Algorithm 2 over vertices classified on the device (reorder.cu: aorder_device): odm[i] /
+// odc[i] = d~ of the i-th memory- / computing-dominated vertex in ascending vertex order
+// (lines 3-4), table[d] = S(d).  Records bucket / rank per placement; the relabel (lines
+// 16-20) runs on the device.
+void aorder_classified(const uint32_t *odm, size_t nmem, const uint32_t *odc, size_t ncomp,
+                       const std::vector<int64_t> &table, int64_t smax, int64_t smin1, int64_t smin2, uint32_t k,
+                       uint32_t *bmem, uint32_t *rmem, uint32_t *bcomp, uint32_t *rcomp,
+                       std::vector<uint32_t> &bucket_off, int64_t &eq3) {
+  AOrderWorkspace &W = workspace();
+  std::lock_guard<std::mutex> lock(W.mu);
+  const double t0 = trace_on() ? now_ms() : 0;
+  double tr[2] = {0, 0};
+  const int64_t *tab = table.data();
+  aorder_greedy(
+      nmem, [&](size_t i) { return tab[odm[i]]; }, ncomp, [&](size_t i) { return tab[odc[i]]; }, smax, smin1, smin2,
+      k, bmem, rmem, bcomp, rcomp, bucket_off, eq3, trace_on() ? tr : nullptr);
+  if (trace_on())
+    fprintf(stderr, "aorder (device-classified) mem=%zu comp=%zu b=%zu: phase1 %.1f ms, phase2 %.1f (bin sorts %.1f)\n",
+            nmem, ncomp, bucket_off.size() - 1, tr[0] - t0, now_ms() - tr[0], tr[1] / 1e6);
 }
 
 std::vector<int64_t> superiority_table(uint32_t maxd, const tc_aorder_params &p) {

@@ -19,6 +19,7 @@ struct tc_graph : tc::Graph {
 namespace tc {
 
 int g_opt_profile = 1;
+int g_opt_aorder_device = 1;
 static thread_local std::string t_err;
 
 void cuda_fail(cudaError_t e, const char *what, const char *file, int line) {
@@ -206,6 +207,8 @@ tc_status tc_set_option(const char *key, int64_t value) {
     } else if (k == "owner_lspan") {
       TC_REQUIRE(value >= 8 && value <= (1 << 24), ST_INVALID, "owner_lspan: 8 .. 2^24");
       g_opt_owner_lspan = (int)value;
+    } else if (k == "aorder_device") {
+      g_opt_aorder_device = value ? 1 : 0;
     } else if (k == "cuckoo") {
       TC_REQUIRE(value >= 0 && value <= 1024, ST_INVALID, "cuckoo: 0 (off) .. 1024 evictions");
       g_opt_cuckoo = (int)value;
@@ -321,8 +324,10 @@ struct BroadcastAOrder : AOrderSource {
     cudaStream_t s = g.stream;
     const uint32_t n = g.n;
     uint64_t hdr[2] = {0, 0};
+    bool on_device = false;  // root: pi already in g.perm (device classification / relabel)
     if (rank == root) {
-      aorder_host(h_od, n, p, h_perm, g.h_bucket_off, g.eq3);
+      on_device = g_opt_aorder_device && aorder_device(g, p);
+      if (!on_device) aorder_host(h_od, n, p, h_perm, g.h_bucket_off, g.eq3);
       hdr[0] = g.h_bucket_off.size();
       hdr[1] = (uint64_t)g.eq3;
     }
@@ -338,9 +343,11 @@ struct BroadcastAOrder : AOrderSource {
       g.h_bucket_off.assign(nb1, 0);
       g.eq3 = (int64_t)hdr[1];
     }
-    if (n) g.perm.alloc(n, s);
-    g.bucket_off.alloc(nb1, s);
-    if (rank == root) {
+    if (!on_device) {
+      if (n) g.perm.alloc(n, s);
+      g.bucket_off.alloc(nb1, s);
+    }
+    if (rank == root && !on_device) {
       if (n) TC_CUDA(cudaMemcpyAsync(g.perm.get(), h_perm, sizeof(uint32_t) * n, cudaMemcpyHostToDevice, s));
       TC_CUDA(cudaMemcpyAsync(g.bucket_off.get(), g.h_bucket_off.data(), sizeof(uint32_t) * nb1,
                               cudaMemcpyHostToDevice, s));

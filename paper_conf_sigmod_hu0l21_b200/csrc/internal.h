@@ -109,6 +109,14 @@ extern std::mutex g_pinned_mu;
 void aorder_units(const std::vector<int64_t> &S, const std::vector<uint8_t> &active, uint32_t k, int order,
                   std::vector<uint32_t> &pos, std::vector<uint32_t> &bucket_off, int64_t &eq3);
 std::vector<int64_t> superiority_table(uint32_t maxd, const tc_aorder_params &p);
+void aorder_classified(const uint32_t *odm, size_t nmem, const uint32_t *odc, size_t ncomp,
+                       const std::vector<int64_t> &table, int64_t smax, int64_t smin1, int64_t smin2, uint32_t k,
+                       uint32_t *bmem, uint32_t *rmem, uint32_t *bcomp, uint32_t *rcomp,
+                       std::vector<uint32_t> &bucket_off, int64_t &eq3);
+// A-order with the classification (lines 3-4) and the relabel (lines 16-20) on the device and
+// the sequential greedy on the host: sets g.perm, g.bucket_off, g.h_bucket_off, g.eq3.
+// Returns false when not applicable (LPT order: host path).
+bool aorder_device(Graph &g, const tc_aorder_params &p);
 // count.cu
 // d_T: optional device accumulator (zeroed by the caller): the count is added there and not
 // read back (returns 0), so a collective can consume it on the stream (tc_count_dist)
@@ -125,6 +133,7 @@ void build_units(Graph &g);  // edge-unit A-order buckets (count.cu)
 
 // options (api.cu)
 extern int g_opt_profile;
+extern int g_opt_aorder_device;  // A-order classification / relabel on the device (1) or host (0)
 extern int g_opt_small_cap;
 extern int g_opt_l2_persist;
 extern int g_opt_bracket;

@@ -223,8 +223,8 @@ void build_oriented_csr(Graph &g) {
 // them for the process lifetime).
 std::mutex g_pinned_mu;
 uint32_t *pinned_u32(size_t n, int slot) {
-  static uint32_t *buf[2] = {nullptr, nullptr};
-  static size_t cap[2] = {0, 0};
+  static uint32_t *buf[8] = {nullptr};
+  static size_t cap[8] = {0};
   if (cap[slot] < n) {
     if (buf[slot]) TC_CUDA(cudaFreeHost(buf[slot]));
     buf[slot] = nullptr;
@@ -233,6 +233,157 @@ uint32_t *pinned_u32(size_t n, int slot) {
     cap[slot] = n;
   }
   return buf[slot];
+}
+
+namespace {
+// ---- A-order classification / relabel on the device (Algorithm 2 lines 3-4 and 16-20)
+constexpr uint32_t AO_SH_BINS = 2048;  // d~ histogram: shared-memory bins, global above
+__global__ void ao_hist_kernel(const uint32_t *__restrict__ od, uint32_t n, uint32_t maxd,
+                               unsigned long long *__restrict__ hist) {
+  __shared__ unsigned s_h[AO_SH_BINS];
+  for (uint32_t i = threadIdx.x; i < AO_SH_BINS; i += blockDim.x) s_h[i] = 0;
+  __syncthreads();
+  for (uint64_t v = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t d = od[v];
+    if (d < AO_SH_BINS) atomicAdd(&s_h[d], 1u);
+    else atomicAdd(&hist[d], 1ull);
+  }
+  __syncthreads();
+  for (uint32_t i = threadIdx.x; i < AO_SH_BINS && i <= maxd; i += blockDim.x)
+    if (s_h[i]) atomicAdd(&hist[i], (unsigned long long)s_h[i]);
+}
+// class flags: fm = memory-dominated (S > 0), fc = computing-dominated (S <= 0), fi = d~ = 0
+__global__ void ao_class_kernel(const uint32_t *__restrict__ od, uint32_t n, const int64_t *__restrict__ tab,
+                                uint32_t *__restrict__ fm, uint32_t *__restrict__ fc, uint32_t *__restrict__ fi) {
+  for (uint64_t v = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t d = od[v];
+    const bool act = d != 0;
+    const bool mem = act && tab[d] > 0;
+    fm[v] = mem;
+    fc[v] = act && !mem;
+    fi[v] = !act;
+  }
+}
+// odm / odc: d~ of the memory- / computing-dominated vertices in ascending vertex order
+__global__ void ao_compact_kernel(const uint32_t *__restrict__ od, uint32_t n, const uint32_t *__restrict__ fm,
+                                  const uint32_t *__restrict__ fc, const uint64_t *__restrict__ pm,
+                                  const uint64_t *__restrict__ pc, uint32_t *__restrict__ odm,
+                                  uint32_t *__restrict__ odc) {
+  for (uint64_t v = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (uint64_t)gridDim.x * blockDim.x) {
+    if (fm[v]) odm[pm[v]] = od[v];
+    else if (fc[v]) odc[pc[v]] = od[v];
+  }
+}
+// pi: bucket start + insertion rank of every placed vertex; inactive vertices last, in id order
+__global__ void ao_relabel_kernel(uint32_t n, const uint32_t *__restrict__ fm, const uint32_t *__restrict__ fc,
+                                  const uint64_t *__restrict__ pm, const uint64_t *__restrict__ pc,
+                                  const uint64_t *__restrict__ pi, const uint32_t *__restrict__ bmem,
+                                  const uint32_t *__restrict__ rmem, const uint32_t *__restrict__ bcomp,
+                                  const uint32_t *__restrict__ rcomp, const uint32_t *__restrict__ boff,
+                                  uint32_t inactive0, uint32_t *__restrict__ perm) {
+  for (uint64_t v = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (uint64_t)gridDim.x * blockDim.x) {
+    uint32_t r;
+    if (fm[v]) {
+      const uint64_t i = pm[v];
+      r = boff[bmem[i]] + rmem[i];
+    } else if (fc[v]) {
+      const uint64_t i = pc[v];
+      r = boff[bcomp[i]] + rcomp[i];
+    } else {
+      r = inactive0 + (uint32_t)pi[v];
+    }
+    perm[v] = r;
+  }
+}
+}  // namespace
+
+bool aorder_device(Graph &g, const tc_aorder_params &p) {
+  if (p.order != 0 || g.n < 2) return false;
+  cudaStream_t s = g.stream;
+  const uint32_t n = g.n;
+  ensure_od(g);
+  const uint32_t maxd = g.max_outdeg;
+  if (maxd > (1u << 24)) return false;  // S per degree value as a table (as aorder_host)
+  const std::vector<int64_t> table = superiority_table(maxd, p);
+  DevBuf<int64_t> dtab;
+  dtab.alloc((size_t)maxd + 1, s);
+  TC_CUDA(cudaMemcpyAsync(dtab.get(), table.data(), sizeof(int64_t) * table.size(), cudaMemcpyHostToDevice, s));
+  DevBuf<unsigned long long> hist;
+  hist.alloc((size_t)maxd + 1, s);
+  TC_CUDA(cudaMemsetAsync(hist.get(), 0, hist.bytes(), s));
+  ao_hist_kernel<<<grid_for(n, 256, 4), 256, 0, s>>>(g.od.get(), n, maxd, hist.get());
+  TC_LAUNCH_CHECK();
+  DevBuf<uint32_t> fm, fc, fi;
+  DevBuf<uint64_t> pm, pc, pi;
+  fm.alloc(n, s);
+  fc.alloc(n, s);
+  fi.alloc(n, s);
+  pm.alloc((uint64_t)n + 1, s);
+  pc.alloc((uint64_t)n + 1, s);
+  pi.alloc((uint64_t)n + 1, s);
+  ao_class_kernel<<<grid_for(n, 256), 256, 0, s>>>(g.od.get(), n, dtab.get(), fm.get(), fc.get(), fi.get());
+  TC_LAUNCH_CHECK();
+  scan_u32_to_u64(fm.get(), pm.get(), n, s);
+  scan_u32_to_u64(fc.get(), pc.get(), n, s);
+  scan_u32_to_u64(fi.get(), pi.get(), n, s);
+  // class sizes and the superiority range from the d~ histogram (S is a function of d~)
+  std::vector<unsigned long long> h(maxd + 1);
+  TC_CUDA(cudaMemcpyAsync(h.data(), hist.get(), sizeof(unsigned long long) * h.size(), cudaMemcpyDeviceToHost, s));
+  TC_CUDA(cudaStreamSynchronize(s));
+  uint64_t nmem = 0, ncomp = 0;
+  int64_t smax = 0, smin1 = INT64_MAX, smin2 = INT64_MAX;
+  for (uint32_t d = 1; d <= maxd; ++d) {
+    if (!h[d]) continue;
+    const int64_t sv = table[d], av = sv < 0 ? -sv : sv;
+    smax = std::max(smax, av);
+    if (sv > 0) {
+      nmem += h[d];
+      smin1 = std::min(smin1, av);
+    } else {
+      ncomp += h[d];
+      if (av) smin2 = std::min(smin2, av);
+    }
+  }
+  DevBuf<uint32_t> odm, odc;
+  odm.alloc(nmem ? nmem : 1, s);
+  odc.alloc(ncomp ? ncomp : 1, s);
+  ao_compact_kernel<<<grid_for(n, 256), 256, 0, s>>>(g.od.get(), n, fm.get(), fc.get(), pm.get(), pc.get(), odm.get(),
+                                                      odc.get());
+  TC_LAUNCH_CHECK();
+  uint32_t *h_odm = pinned_u32(nmem ? nmem : 1, 2), *h_odc = pinned_u32(ncomp ? ncomp : 1, 3);
+  uint32_t *h_bm = pinned_u32(nmem ? nmem : 1, 4), *h_rm = pinned_u32(nmem ? nmem : 1, 5);
+  uint32_t *h_bc = pinned_u32(ncomp ? ncomp : 1, 6), *h_rc = pinned_u32(ncomp ? ncomp : 1, 7);
+  if (nmem) TC_CUDA(cudaMemcpyAsync(h_odm, odm.get(), 4 * nmem, cudaMemcpyDeviceToHost, s));
+  if (ncomp) TC_CUDA(cudaMemcpyAsync(h_odc, odc.get(), 4 * ncomp, cudaMemcpyDeviceToHost, s));
+  TC_CUDA(cudaStreamSynchronize(s));
+  // lines 1-15 on the host (sequential greedy)
+  aorder_classified(h_odm, nmem, h_odc, ncomp, table, smax, smin1, smin2, p.k, h_bm, h_rm, h_bc, h_rc,
+                    g.h_bucket_off, g.eq3);
+  // lines 16-20 on the device
+  DevBuf<uint32_t> bm, rm, bc, rc;
+  bm.alloc(nmem ? nmem : 1, s);
+  rm.alloc(nmem ? nmem : 1, s);
+  bc.alloc(ncomp ? ncomp : 1, s);
+  rc.alloc(ncomp ? ncomp : 1, s);
+  if (nmem) {
+    TC_CUDA(cudaMemcpyAsync(bm.get(), h_bm, 4 * nmem, cudaMemcpyHostToDevice, s));
+    TC_CUDA(cudaMemcpyAsync(rm.get(), h_rm, 4 * nmem, cudaMemcpyHostToDevice, s));
+  }
+  if (ncomp) {
+    TC_CUDA(cudaMemcpyAsync(bc.get(), h_bc, 4 * ncomp, cudaMemcpyHostToDevice, s));
+    TC_CUDA(cudaMemcpyAsync(rc.get(), h_rc, 4 * ncomp, cudaMemcpyHostToDevice, s));
+  }
+  g.bucket_off.alloc(g.h_bucket_off.size(), s);
+  TC_CUDA(cudaMemcpyAsync(g.bucket_off.get(), g.h_bucket_off.data(), sizeof(uint32_t) * g.h_bucket_off.size(),
+                          cudaMemcpyHostToDevice, s));
+  g.perm.alloc(n, s);
+  ao_relabel_kernel<<<grid_for(n, 256), 256, 0, s>>>(n, fm.get(), fc.get(), pm.get(), pc.get(), pi.get(), bm.get(),
+                                                      rm.get(), bc.get(), rc.get(), g.bucket_off.get(),
+                                                      g.h_bucket_off.back(), g.perm.get());
+  TC_LAUNCH_CHECK();
+  TC_CUDA(cudaStreamSynchronize(s));  // pinned buffers are reused by the next A-order
+  g.identity_perm = false;
+  return true;
 }
 
 void reorder_graph(Graph &g, int rule, const tc_aorder_params &p, AOrderSource *src) {
@@ -262,6 +413,12 @@ void reorder_graph(Graph &g, int rule, const tc_aorder_params &p, AOrderSource *
     // d~ down and pi up through pinned staging buffers (kept across calls, one A-order at a
     // time: the host greedy holds the lock anyway)
     std::lock_guard<std::mutex> lock(g_pinned_mu);
+    if (!src && g_opt_aorder_device && aorder_device(g, p)) {
+      g.reorder_rule = rule;
+      build_oriented_csr(g);
+      g.state = G_ORDERED;
+      return;
+    }
     uint32_t *h_od = pinned_u32(n ? n : 1, 0), *h_perm = pinned_u32(n ? n : 1, 1);
     if (n) TC_CUDA(cudaMemcpyAsync(h_od, g.od.get(), sizeof(uint32_t) * n, cudaMemcpyDeviceToHost, s));
     TC_CUDA(cudaStreamSynchronize(s));
