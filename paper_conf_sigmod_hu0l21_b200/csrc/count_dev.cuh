@@ -38,7 +38,10 @@ constexpr int TS_L = TC_TS_L;         // CTA items (pieces): the table's size in
 #define TC_TS_LMAX 4
 #endif
 constexpr int TS_LMAX = TC_TS_LMAX;
-constexpr uint32_t LG_SMEM_WORDS = (PIECE + 72) + ((PIECE << TS_L) + 64) / 2;  // piece (+pad) + u16 table
+#ifndef TC_LG_SMEM_WORDS
+#define TC_LG_SMEM_WORDS ((PIECE + 72) + ((PIECE << TS_L) + 64) / 2)
+#endif
+constexpr uint32_t LG_SMEM_WORDS = TC_LG_SMEM_WORDS;  // piece (+pad) + u16 table / the cuckoo tables
 constexpr uint32_t CHUNK = 8;         // worklist entries per atomic fetch
 constexpr uint32_t CK_MAXL = (PIECE * 9) / 10;  // cuckoo sets: pieces up to 0.9 x 4096 (2 x 4096 slots)
 

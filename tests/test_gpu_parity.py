@@ -238,6 +238,30 @@ def test_aorder_params_bw_table_and_lpt():
     g.free()
 
 
+@pytest.mark.parametrize("device_side", [0, 1])
+def test_aorder_host_and_device_classification(device_side):
+    """A-order with the classification / relabel on the host (aorder_device=0) and on the
+    device (1): pi, bucket_off and Eq.3 equal the oracle's, incl. a BW table, k != 32 and
+    graphs with isolated vertices."""
+    tc.tc_set_option("aorder_device", device_side)
+    try:
+        for seed, (sc, ef, d, k, lam, bw) in enumerate(((12, 16, "degree", 32, 9.682, None),
+                                                       (11, 8, "paper", 16, 3.0, np.linspace(1.0, 50.0, 64)),
+                                                       (13, 4, "id", 7, 9.682, None))):
+            spec = graphgen.rmat_spec(sc, ef, 400 + seed)
+            src, dst = graphgen.generate_cpu(spec)
+            ref = oracle.run(src, dst, spec.n, d, "paper", k=k, lam=lam, bw=bw)
+            g = tc.Graph(src, dst, spec.n).direct(d).reorder("paper", k=k, lam=lam, bw=bw)
+            offs, col, perm = g.export()
+            assert np.array_equal(perm, ref["perm"]), (seed, device_side)
+            assert np.array_equal(g.export_buckets(), ref["bucket_off"]), (seed, device_side)
+            assert g.stats()["eq3"] == oracle.objective_eq3(ref["bucket_off"], ref["perm"], ref["od"], lam=lam, bw=bw)
+            assert g.count() == ref["T"]
+            g.free()
+    finally:
+        tc.tc_set_option("aorder_device", 1)
+
+
 def test_gpu_generator_matches_cpu():
     import torch
     for spec in (graphgen.rmat_spec(16, 4, 11), graphgen.er_spec(100003, 1 << 18, 12)):
