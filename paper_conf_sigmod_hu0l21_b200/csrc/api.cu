@@ -196,6 +196,7 @@ tc_status tc_set_option(const char *key, int64_t value) {
       g_opt_intersect = (int)value;
     }
     else if (k == "peel_coop") g_opt_peel_coop = value ? 1 : 0;
+    else if (k == "peel_red") g_opt_peel_red = value < 0 ? -1 : (value ? 1 : 0);
     else if (k == "split") g_opt_split = value ? 1 : 0;
     else if (k == "shorter") g_opt_shorter = value ? 1 : 0;
     else if (k == "owner_span") {

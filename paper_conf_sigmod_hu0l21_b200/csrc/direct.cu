@@ -26,6 +26,7 @@
 namespace tc {
 
 int g_opt_peel_coop = 1;  // whole A-direction peel in one cooperative launch
+int g_opt_peel_red = -1;  // coop peel: decrements as RED + frontier scan (1), returning atomics (0), auto (-1)
 
 namespace {
 
@@ -106,9 +107,17 @@ __global__ void mark_kernel(const uint32_t *__restrict__ F, unsigned nf, uint8_t
 }
 
 // Decrement of one incident edge (v, nbr) of a frontier vertex (Algorithm 1 line 12-16).
+// RED = true (the cooperative peel): a fire-and-forget reduction (the warp does not wait
+// for the returned value); the vertices that crossed the threshold are found afterwards by
+// a scan of the unpeeled vertices (res <= thr), the same set as the crossing test below
+template <bool RED = false>
 __device__ __forceinline__ bool expand_one(uint32_t nbr, const uint8_t *__restrict__ state, uint32_t *res,
                                            uint64_t thr) {
   if (state[nbr] != V_UNPEELED) return false;
+  if (RED) {
+    atomicSub(&res[nbr], 1u);  // result unused: compiled to RED
+    return false;
+  }
   const uint32_t old = atomicSub(&res[nbr], 1u);
   return (uint64_t)old == thr + 1;
 }
@@ -185,6 +194,7 @@ __global__ void expand_kernel(const uint32_t *__restrict__ F, const unsigned *__
 // memory and binary-searches it per chunk; with more than HUB_MAX hubs the hubs are taken
 // one after another, each spread over every thread of the grid.  Called by whole CTAs.
 constexpr uint32_t HUB_CHUNK = 1024, HUB_MAX = 8192;
+template <bool RED = false>
 __device__ __forceinline__ void expand_hubs(const uint32_t *__restrict__ F, unsigned nh,
                                             const uint64_t *__restrict__ soffs, const uint32_t *__restrict__ sadj,
                                             const uint8_t *__restrict__ state, uint32_t *res, uint64_t thr,
@@ -203,7 +213,7 @@ __device__ __forceinline__ void expand_hubs(const uint32_t *__restrict__ F, unsi
         uint32_t nbr = 0;
         if (p < e) {
           nbr = sadj[p];
-          cross = expand_one(nbr, state, res, thr);
+          cross = expand_one<RED>(nbr, state, res, thr);
         }
         warp_append(cross, nbr, next, nnext);
       }
@@ -253,7 +263,7 @@ __device__ __forceinline__ void expand_hubs(const uint32_t *__restrict__ F, unsi
       uint32_t nbr = 0;
       if (p < ce) {
         nbr = sadj[p];
-        cross = expand_one(nbr, state, res, thr);
+        cross = expand_one<RED>(nbr, state, res, thr);
       }
       warp_append(cross, nbr, next, nnext);
     }
@@ -289,6 +299,7 @@ struct PeelArgs {
   uint32_t *out;      // [0] levels, [1] subrounds, [2] error
   uint32_t n;
   uint64_t m;
+  int red;            // residual-degree decrements as RED + a scan for the next frontier
 };
 
 __global__ __launch_bounds__(256) void peel_coop_kernel(PeelArgs A) {
@@ -369,7 +380,7 @@ __global__ __launch_bounds__(256) void peel_coop_kernel(PeelArgs A) {
           uint32_t nbr = 0;
           if (j < total) {
             nbr = A.sadj[ao + (j - eo)];
-            cross = expand_one(nbr, A.state, A.res, thr);
+            cross = A.red ? expand_one<true>(nbr, A.state, A.res, thr) : expand_one<false>(nbr, A.state, A.res, thr);
           }
           warp_append(cross, nbr, next, cnext);
         }
@@ -384,17 +395,25 @@ __global__ __launch_bounds__(256) void peel_coop_kernel(PeelArgs A) {
           uint32_t nbr = 0;
           if (p < e) {
             nbr = A.sadj[p];
-            cross = expand_one(nbr, A.state, A.res, thr);
+            cross = A.red ? expand_one<true>(nbr, A.state, A.res, thr) : expand_one<false>(nbr, A.state, A.res, thr);
           }
           warp_append(cross, nbr, next, cnext);
         }
       }
       // hubs: chunks of HUB_CHUNK edges over every warp of the grid
-      expand_hubs(A.Fh, nh, A.soffs, A.sadj, A.state, A.res, thr, next, cnext, s_pre);
+      if (A.red) expand_hubs<true>(A.Fh, nh, A.soffs, A.sadj, A.state, A.res, thr, next, cnext, s_pre);
+      else expand_hubs<false>(A.Fh, nh, A.soffs, A.sadj, A.state, A.res, thr, next, cnext, s_pre);
       grid.sync();
       // peel the frontier (Algorithm 1 line 17-18); reset the split counters and the
       // next-frontier counter of the following subround
       for (uint64_t i = gtid; i < nf; i += gthreads) A.state[F[i]] = V_PEELED;
+      if (A.red) {  // next frontier: the unpeeled vertices whose residual degree reached thr
+        for (uint64_t base = gtid & ~31ull; base < n; base += gthreads) {
+          const uint64_t v = base + lane;
+          const bool want = v < n && A.state[v] == V_UNPEELED && (uint64_t)A.res[v] <= thr;
+          warp_append(want, (uint32_t)v, next, cnext);
+        }
+      }
       if (gtid == 0) {
         A.ctr[4] = A.ctr[5] = A.ctr[6] = 0;
         A.ctr[2 + ((r + 1) & 1)] = 0;
@@ -511,7 +530,10 @@ void peel_paper(Graph &g) {
       TC_CUDA(cudaMemsetAsync(out.get(), 0, 3 * sizeof(uint32_t), s));
       TC_CUDA(cudaMemsetAsync(counters.get(), 0, counters.bytes(), s));
       PeelArgs A{soffs.get(), sadj.get(), g.deg.get(), res.get(), g.sub.get(), g.dsnap.get(), state.get(),
-                 F.get(), next.get(), Fs.get(), Fb.get(), Fh.get(), counters.get(), out.get(), n, m};
+                 F.get(), next.get(), Fs.get(), Fb.get(), Fh.get(), counters.get(), out.get(), n, m,
+                 // auto: RED from 2^25 vertices (the frontier scan costs n per subround; the
+                 // waits on returning atomics to hubs dominate only on large graphs)
+                 g_opt_peel_red >= 0 ? g_opt_peel_red : (n >= (1u << 25) ? 1 : 0)};
       void *args[] = {&A};
       {
         ProfScope prof("peel", s, 0.0);

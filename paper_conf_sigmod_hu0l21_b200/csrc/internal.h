@@ -140,6 +140,7 @@ extern int g_opt_bracket;
 extern int g_opt_lean;  // register-lean count_small instantiations
 extern int g_opt_extra;  // §5.3 experiment: extra searches per wedge (-1 = production kernel)
 extern int g_opt_intersect;  // 0 binary search, 1 sort-merge (count only)
+extern int g_opt_peel_red;   // coop peel: RED decrements + frontier scan (1/0, -1 auto)
 extern int g_opt_peel_coop;  // A-direction peel as one cooperative launch
 extern int g_opt_split;  // orientation split CSR build (original labels)
 extern int g_opt_shorter;      // shorter-list owner schedule for count modes

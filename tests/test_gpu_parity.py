@@ -262,6 +262,27 @@ def test_aorder_host_and_device_classification(device_side):
         tc.tc_set_option("aorder_device", 1)
 
 
+@pytest.mark.parametrize("red", [0, 1])
+def test_adirection_peel_red_and_atomic(red):
+    """A-direction peel with returning atomics (crossing test per decrement) and with RED
+    decrements + a frontier scan: sub / dsnap / d~ and T equal the oracle's (Alg.1)."""
+    tc.tc_set_option("peel_red", red)
+    try:
+        for seed, (sc, ef) in enumerate(((12, 16), (13, 8), (10, 48))):
+            spec = graphgen.rmat_spec(sc, ef, 600 + seed)
+            src, dst = graphgen.generate_cpu(spec)
+            ref = oracle.run(src, dst, spec.n, "paper", "none")
+            g = tc.Graph(src, dst, spec.n).direct("paper")
+            od, sub, dsnap = g.export_direct(internals=True)
+            info = ref["direct_info"]
+            assert np.array_equal(sub, info["sub"]) and np.array_equal(dsnap, info["dsnap"]), (seed, red)
+            assert np.array_equal(od, ref["od"]), (seed, red)
+            assert g.count() == ref["T"]
+            g.free()
+    finally:
+        tc.tc_set_option("peel_red", -1)
+
+
 def test_gpu_generator_matches_cpu():
     import torch
     for spec in (graphgen.rmat_spec(16, 4, 11), graphgen.er_spec(100003, 1 << 18, 12)):
