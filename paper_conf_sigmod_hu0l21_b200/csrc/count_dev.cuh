@@ -19,6 +19,9 @@ constexpr int LG_THREADS = 256;       // large kernel: 8 warps
 constexpr int LG_WARPS = LG_THREADS / 32;
 constexpr uint32_t PIECE = 4096;      // large kernel: N+(u) piece in shared memory (16 KB)
 constexpr uint32_t LG_SUB = 8;        // large kernel: v's per dynamically fetched sub-chunk
+#ifndef TC_LG_NB
+#define TC_LG_NB 8                    // large kernel, count: 32-wedge steps per gather block
+#endif
 #ifndef TC_LG_SUB_OWN
 #define TC_LG_SUB_OWN 32
 #endif
@@ -387,7 +390,9 @@ __device__ __forceinline__ uint32_t wedge_loop(const uint32_t *__restrict__ col,
     }
   };
   uint32_t st = 0;
-  if (NB == 8)  // CTA items (register budget 48): 8 gathers in flight per lane
+  if (NB == 16)  // (variant: 16 gathers in flight per lane)
+    for (; st + 16 <= steps; st += 16) block(std::integral_constant<int, 16>(), st);
+  if (NB >= 8)  // CTA items (register budget 48): 8 gathers in flight per lane
     for (; st + 8 <= steps; st += 8) block(std::integral_constant<int, 8>(), st);
   for (; st + 4 <= steps; st += 4) block(std::integral_constant<int, 4>(), st);
   if (st + 2 <= steps) {
@@ -884,7 +889,7 @@ __global__ __launch_bounds__(LG_THREADS, OWN ? TC_LG_MINB_OWN : 5) void count_la
         if (c0 >= cend) break;
         const bool valid = lane_id() < SUB && c0 + lane_id() < cend;
         const uint32_t v = valid ? ldg_u32(olist + c0 + lane_id()) : 0u;
-        cnt += warp_chunk<MODE, MODE == 0 ? 8 : 4, true>(offs, col, v, valid, list, shift, S2 >= 0 ? tbase : 0xffffffffu, 0xffffffffu, plen,
+        cnt += warp_chunk<MODE, MODE == 0 ? TC_LG_NB : 4, true>(offs, col, v, valid, list, shift, S2 >= 0 ? tbase : 0xffffffffu, 0xffffffffu, plen,
                                 true, lo, hi, ws, tv, c0 + lane_id(), a, a + p0, vbits, S2 >= 0 ? S2 : -2, sh,
                                 abs_t ? 1 : 0, ck_sh);
       }
