@@ -242,7 +242,9 @@ tc_status tc_export_units(tc_graph *g, uint64_t *units, uint32_t *unit_off);
  * falls back to the sorted piece, counts are unchanged), "aorder_device" (1 = default: the
  * A-order classification into memory- / computing-dominated vertices (Alg.2 lines 3-4) and
  * the relabel (lines 16-20) run on the device around the host's sequential greedy; 0 = all
- * on the host; identical pi). */
+ * on the host; identical pi), "e2sort" (shorter-list schedule: the owners an edge gives
+ * to the endpoint with the longer list grouped by a radix sort of (x, u) pairs instead of
+ * per-x cursor atomics; -1 = auto (from 2^28 edges), 0 / 1). */
 tc_status tc_set_option(const char *key, int64_t value);
 
 /* Per-kernel profile since the last reset, as JSON text into buf (host, cap bytes):

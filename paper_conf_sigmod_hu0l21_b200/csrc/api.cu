@@ -213,6 +213,8 @@ tc_status tc_set_option(const char *key, int64_t value) {
     } else if (k == "cuckoo") {
       TC_REQUIRE(value >= 0 && value <= 1024, ST_INVALID, "cuckoo: 0 (off) .. 1024 evictions");
       g_opt_cuckoo = (int)value;
+    } else if (k == "e2sort") {
+      g_opt_e2sort = value < 0 ? -1 : (value ? 1 : 0);
     } else if (k == "otiles") {
       TC_REQUIRE(value >= 0 && value <= 255, ST_INVALID, "otiles: 0 (auto) .. 255");
       g_opt_otiles = (int)value;

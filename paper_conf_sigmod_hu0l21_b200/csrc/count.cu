@@ -43,6 +43,7 @@ int g_opt_owner_span = 128;  // owners per warp item (shorter-list schedule)
 int g_opt_owner_lspan = 2048;  // owners per CTA item
 int g_opt_vtiles = 1;        // classic count: streamed lists in this many L2 label tiles (1 = off)
 int g_opt_cuckoo = 64;       // count-only CTA items: cuckoo set of the staged piece, max evictions (0 = off)
+int g_opt_e2sort = -1;       // E2 owners grouped by a sort (no returning cursor atomics); -1 auto
 int g_opt_otiles = 1;        // shorter-list CTA items: owner-label L2 tiles (0 = auto, 1 = off; default off: measured no faster)
 int g_opt_otile_mb = 48;     // auto: MB of col per owner-label tile
 int g_opt_otile_min = 4;     // a large x is tiled when it has >= otile_min * tiles owners
@@ -176,7 +177,7 @@ __global__ void owners_count_kernel(const uint64_t *__restrict__ offs, const uin
                                     const uint32_t *__restrict__ od, uint32_t ub, uint32_t ue,
                                     uint32_t *__restrict__ e1c, uint32_t *__restrict__ e2c,
                                     const uint32_t *__restrict__ lg, const uint32_t *__restrict__ bnd, uint32_t nt,
-                                    uint32_t *__restrict__ tcnt) {
+                                    uint32_t *__restrict__ tcnt, uint32_t *__restrict__ e2s) {
   __shared__ uint32_t s_bnd[MAX_OTILES + 1];
   if (tcnt) stage_bounds(s_bnd, bnd, nt);
   const uint64_t nw = (uint64_t)gridDim.x * (blockDim.x / 32);
@@ -185,7 +186,7 @@ __global__ void owners_count_kernel(const uint64_t *__restrict__ offs, const uin
     const uint32_t du = (uint32_t)(offs[u + 1] - a);
     if (du < 2) continue;
     const uint32_t lu = tcnt ? lg[u] : 0xffffffffu;  // warp-uniform
-    uint32_t c1 = 0;
+    uint32_t c1 = 0, c2 = 0;
     for (uint32_t j0 = 0; j0 < du; j0 += 32) {
       const uint32_t j = j0 + lane_id();
       uint32_t v = 0, dv = 0;
@@ -195,6 +196,7 @@ __global__ void owners_count_kernel(const uint64_t *__restrict__ offs, const uin
       }
       const bool e1 = j < du && dv >= 1 && dv <= du;
       c1 += __popc(__ballot_sync(0xffffffffu, e1));
+      c2 += __popc(__ballot_sync(0xffffffffu, j < du && dv > du));
       if (lu != 0xffffffffu) warp_agg_add(e1, e1 ? tile_of(s_bnd, nt, v) : 0u, tcnt + (uint64_t)lu * nt);
       if (j < du && dv > du) {
         atomicAdd(&e2c[v], 1u);
@@ -204,7 +206,10 @@ __global__ void owners_count_kernel(const uint64_t *__restrict__ offs, const uin
         }
       }
     }
-    if (lane_id() == 0) e1c[u] = c1;
+    if (lane_id() == 0) {
+      e1c[u] = c1;
+      if (e2s) e2s[u] = c2;
+    }
   }
 }
 // per large x: tiled iff it has >= tmin owners (else lg[x] = ~0: untiled); tiled rows get
@@ -326,6 +331,50 @@ __global__ void owners_scatter_kernel(const uint64_t *__restrict__ offs, const u
           own[atomicAdd(&e2cur[v], 1ull)] = (uint32_t)u;
       }
     }
+  }
+}
+
+// E2 owners grouped by a sort instead of returning cursor atomics (option "e2sort"): the
+// cursor of a hub x takes every E2 owner of x, and the returned positions serialise there.
+// e2s[u] = #E2 edges of source u (owners_count); the E1 scatter also writes the E2 pairs
+// (x << vbits) | u compactly at e2pos[u]; an LSD sort on the x bits groups them (stable);
+// the placement puts the j-th pair of x at own[ooff[x] + e1c[x] + j].
+__global__ void owners_scatter_e2keys_kernel(const uint64_t *__restrict__ offs, const uint32_t *__restrict__ col,
+                                             const uint32_t *__restrict__ od, uint32_t ub, uint32_t ue,
+                                             const uint64_t *__restrict__ ooff, const uint64_t *__restrict__ e2pos,
+                                             uint32_t vbits, uint32_t *__restrict__ own, uint64_t *__restrict__ keys) {
+  const uint64_t nw = (uint64_t)gridDim.x * (blockDim.x / 32);
+  for (uint64_t u = ub + (uint64_t)blockIdx.x * (blockDim.x / 32) + warp_id(); u < ue; u += nw) {
+    const uint64_t a = offs[u];
+    const uint32_t du = (uint32_t)(offs[u + 1] - a);
+    if (du < 2) continue;
+    uint64_t p1 = ooff[u], p2 = e2pos[u];
+    for (uint32_t j0 = 0; j0 < du; j0 += 32) {
+      const uint32_t j = j0 + lane_id();
+      uint32_t v = 0, dv = 0;
+      if (j < du) {
+        v = col[a + j];
+        dv = od[v];
+      }
+      const bool e1 = j < du && dv >= 1 && dv <= du;
+      const bool e2 = j < du && dv > du;
+      const unsigned lt = (1u << lane_id()) - 1u;
+      const unsigned m1 = __ballot_sync(0xffffffffu, e1), m2 = __ballot_sync(0xffffffffu, e2);
+      if (e1) own[p1 + __popc(m1 & lt)] = v;
+      if (e2) keys[p2 + __popc(m2 & lt)] = ((uint64_t)v << vbits) | u;
+      p1 += __popc(m1);
+      p2 += __popc(m2);
+    }
+  }
+}
+__global__ void owners_place_e2_kernel(const uint64_t *__restrict__ sorted, uint64_t total, uint32_t vbits,
+                                       const uint64_t *__restrict__ ooff, const uint32_t *__restrict__ e1c,
+                                       const uint64_t *__restrict__ e2start, uint32_t *__restrict__ own) {
+  const uint64_t mask = (1ull << vbits) - 1;
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < total; i += (uint64_t)gridDim.x * blockDim.x) {
+    const uint64_t key = sorted[i];
+    const uint64_t x = key >> vbits;
+    own[ooff[x] + e1c[x] + (i - e2start[x])] = (uint32_t)(key & mask);
   }
 }
 
@@ -861,9 +910,22 @@ uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *
           nlaunch += 4;
         }
         const unsigned wgrid = grid_for((uint64_t)(ue - ub) * 32, 256, 8);
+        // auto: from 2^28 edges (configs[3] count -3.4 ms, configs[4] -33 ms; R-MAT s22 +0.5 ms)
+        const bool e2sort = (g_opt_e2sort < 0 ? g.m >= (1ull << 28) : g_opt_e2sort != 0) && !nt && 2 * vbits <= 64;
+        DevBuf<uint32_t> e2s;  // E2 edges per source (e2sort)
+        if (e2sort) {
+          e2s.alloc(n, s);
+          TC_CUDA(cudaMemsetAsync(e2s.get(), 0, e2s.bytes(), s));
+        }
         owners_count_kernel<<<wgrid, 256, 0, s>>>(g.offs.get(), g.col.get(), od_new.get(), ub, ue, e1c.get(),
-                                                  e2c.get(), lg.get(), bnd.get(), nt, nt ? tcnt.get() : nullptr);
+                                                  e2c.get(), lg.get(), bnd.get(), nt, nt ? tcnt.get() : nullptr,
+                                                  e2sort ? e2s.get() : nullptr);
         TC_LAUNCH_CHECK();
+        DevBuf<uint64_t> e2start;
+        if (e2sort) {  // group starts of the E2 owners, before e2c becomes the total count
+          e2start.alloc((uint64_t)n + 1, s);
+          scan_u32_to_u64(e2c.get(), e2start.get(), n, s);
+        }
         owners_total_kernel<<<grid_for(n, 256), 256, 0, s>>>(e1c.get(), n, e2c.get());
         TC_LAUNCH_CHECK();
         scan_u32_to_u64(e2c.get(), ooff.get(), n, s);
@@ -877,10 +939,32 @@ uint64_t count_graph(Graph &g, uint32_t ub, uint32_t ue, uint64_t *d_tv, float *
           TC_LAUNCH_CHECK();
           ++nlaunch;
         }
-        owners_scatter_kernel<<<wgrid, 256, 0, s>>>(g.offs.get(), g.col.get(), od_new.get(), ub, ue, ooff.get(),
-                                                    e2cur.get(), own.get(), lg.get(), bnd.get(), nt,
-                                                    nt ? tcnt.get() : nullptr);
-        TC_LAUNCH_CHECK();
+        if (e2sort) {
+          DevBuf<uint64_t> e2pos;
+          e2pos.alloc((uint64_t)n + 1, s);
+          scan_u32_to_u64(e2s.get(), e2pos.get(), n, s);
+          uint64_t total = 0;
+          TC_CUDA(cudaMemcpyAsync(&total, e2pos.get() + n, sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
+          TC_CUDA(cudaStreamSynchronize(s));
+          DevBuf<uint64_t> k2, t2;
+          k2.alloc(total ? total : 1, s);
+          t2.alloc(total ? total : 1, s);
+          owners_scatter_e2keys_kernel<<<wgrid, 256, 0, s>>>(g.offs.get(), g.col.get(), od_new.get(), ub, ue,
+                                                             ooff.get(), e2pos.get(), vbits, own.get(), k2.get());
+          TC_LAUNCH_CHECK();
+          if (total) {
+            const uint64_t *sorted = radix_sort_u64(k2.get(), t2.get(), total, (int)vbits, (int)(2 * vbits), s);
+            owners_place_e2_kernel<<<grid_for(total, 256), 256, 0, s>>>(sorted, total, vbits, ooff.get(), e1c.get(),
+                                                                       e2start.get(), own.get());
+            TC_LAUNCH_CHECK();
+          }
+          nlaunch += 5;
+        } else {
+          owners_scatter_kernel<<<wgrid, 256, 0, s>>>(g.offs.get(), g.col.get(), od_new.get(), ub, ue, ooff.get(),
+                                                      e2cur.get(), own.get(), lg.get(), bnd.get(), nt,
+                                                      nt ? tcnt.get() : nullptr);
+          TC_LAUNCH_CHECK();
+        }
         nlaunch += 6;
         ow = Owners{ooff.get(), own.get(), (uint32_t)g_opt_owner_span, (uint32_t)g_opt_owner_lspan, 0, 0xffffffffu};
         if (nt) {

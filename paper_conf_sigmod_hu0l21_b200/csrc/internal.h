@@ -148,6 +148,7 @@ extern int g_opt_owner_span;   // owners per warp item
 extern int g_opt_owner_lspan;  // owners per CTA item
 extern int g_opt_vtiles;       // classic count: label tiles of the streamed lists (1 = off)
 extern int g_opt_cuckoo;       // count-only CTA items: cuckoo hash set of the staged piece
+extern int g_opt_e2sort;       // E2 owners grouped by a sort instead of cursor atomics
 extern int g_opt_otiles;       // shorter-list CTA items: owner-label L2 tiles (0 = auto, 1 = off)
 extern int g_opt_otile_mb;     // auto: MB of col per owner tile
 extern int g_opt_otile_min;    // tiled x: >= otile_min * tiles owners

@@ -585,6 +585,28 @@ def test_cuckoo_piece_sets(evictions):
         tc.tc_set_option("small_cap", 256)
 
 
+@pytest.mark.parametrize("e2sort", [0, 1])
+def test_owner_e2_grouping_sort_and_atomics(e2sort):
+    """E2 owners grouped by cursor atomics (0) or by a sort of the (x, u) pairs (1): T equal
+    to the oracle's, whole and on work-balanced slices (the owners of a slice's sources)."""
+    tc.tc_set_option("e2sort", e2sort)
+    tc.tc_set_option("small_cap", 32)
+    try:
+        for seed, (sc, ef, d, r) in enumerate(((13, 32, "degree", "paper"), (12, 16, "paper", "none"),
+                                               (12, 8, "id", "degree"))):
+            spec = graphgen.rmat_spec(sc, ef, 990 + seed)
+            src, dst = graphgen.generate_cpu(spec)
+            ref = oracle.run(src, dst, spec.n, d, r)
+            g = tc.Graph(src, dst, spec.n).direct(d).reorder(r)
+            assert g.count() == ref["T"], (seed, e2sort)
+            b = g.partition(4).tolist()
+            assert sum(g.count_range(a, c) for a, c in zip(b, b[1:])) == ref["T"], (seed, e2sort)
+            g.free()
+    finally:
+        tc.tc_set_option("e2sort", -1)
+        tc.tc_set_option("small_cap", 256)
+
+
 def test_extra_compute_instrumented_kernel_counts_unchanged():
     """The §5.3 balance-point instrumentation (option extra_compute, MODE 3: p_c extra
     searches per wedge, results discarded) leaves T and t(v) equal to the oracle's."""
