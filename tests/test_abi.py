@@ -52,3 +52,30 @@ def test_no_cpu_fallback_without_gpu():
         tc.Graph(z, z[::-1].copy(), 2)
     assert e.value.status == tc.TC_ERR_CUDA
     assert "no CUDA device" in str(e.value)
+
+
+# (key, default, an accepted value, a rejected value or None): the options tc.h documents
+OPTIONS = [("cuckoo", 64, 0, 2000), ("otiles", 1, 7, 300), ("otile_mb", 48, 16, 0), ("otile_min", 4, 0, -1),
+           ("e2sort", -1, 1, None), ("aorder_device", 1, 0, None), ("peel_red", -1, 1, None),
+           ("owner_span", 128, 32, None), ("owner_lspan", 2048, 64, 4), ("small_cap", 256, 512, 100),
+           ("extra_compute", -1, 8, 2000), ("shorter", 1, 0, None), ("vtiles", 1, 2, 0)]
+
+
+@pytest.mark.parametrize("key,default,good,bad", OPTIONS, ids=[o[0] for o in OPTIONS])
+def test_options_validate_and_restore(key, default, good, bad):
+    """tc_set_option accepts the documented range, rejects values outside it with
+    TC_ERR_INVALID (no partial state), and unknown keys; runs without a GPU."""
+    try:
+        tc.tc_set_option(key, good)
+        if bad is not None:
+            with pytest.raises(tc.TCError) as e:
+                tc.tc_set_option(key, bad)
+            assert e.value.status == tc.TC_ERR_INVALID
+    finally:
+        tc.tc_set_option(key, default)
+
+
+def test_unknown_option_rejected():
+    with pytest.raises(tc.TCError) as e:
+        tc.tc_set_option("no_such_option", 1)
+    assert e.value.status == tc.TC_ERR_INVALID
