@@ -216,7 +216,10 @@ tc_status tc_export_units(tc_graph *g, uint64_t *units, uint32_t *unit_off);
  * per barrier-closed superstep, the kernel of Fig.13; 1 and 2 apply to
  * tc_count / tc_count_range / tc_count_dist without per-vertex output), "peel_coop" (0/1:
  * run the whole A-direction peel as one cooperative launch with grid-wide barriers instead
- * of 5 launches and a host round trip per subround, default 1), "lean" (0/1: when every
+ * of 5 launches and a host round trip per subround, default 1), "peel_red" (-1 = auto, the
+ * default: from 2^25 vertices the cooperative peel decrements residual degrees with
+ * fire-and-forget reductions and finds the next frontier by a scan of the unpeeled
+ * vertices, the same set as the per-decrement crossing test of Alg.1; 0 / 1 force it), "lean" (0/1: when every
  * warp-item list of a count has < 32 entries, run the 32-register short-list instantiation
  * of the warp-item kernel, 8 CTAs per SM; default 1), "trim_memory" (any
  * value: release the library's cached device blocks), "extra_compute" (-1 = off, the
