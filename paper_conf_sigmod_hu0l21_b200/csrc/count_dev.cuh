@@ -23,7 +23,7 @@ constexpr uint32_t LG_SUB = 8;        // large kernel: v's per dynamically fetch
 #define TC_LG_NB 8                    // large kernel, count: 32-wedge steps per gather block
 #endif
 #ifndef TC_LG_SUB_OWN
-#define TC_LG_SUB_OWN 32
+#define TC_LG_SUB_OWN 16
 #endif
 constexpr uint32_t LG_SUB_OWN = TC_LG_SUB_OWN;  // ... of the shorter-list schedule (owners)
 #ifndef TC_LG_MINB_OWN
